@@ -1,0 +1,355 @@
+"""Pins for the oracle's converters, merge-path coordinates, CSR5 encoding,
+features and partition, CPU only."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import matgen
+import oracle
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def load(name):
+    with open(os.path.join(GOLD, name)) as f:
+        return json.load(f)
+
+
+def csr_of(g):
+    return matgen.HostCSR(np.array(g["row_ptr"], np.int64), np.array(g["col"], np.int32),
+                          np.array(g["val"], np.float64), g["n_rows"], g["n_cols"])
+
+
+def structured_cases():
+    """Small matrices with empty rows (leading/trailing/runs), long rows, runs of
+    consecutive columns, rectangular shapes."""
+    out = [csr_of(load("app_a_4x4.json")), csr_of(load("app_a_5x5.json"))]
+    out.append(matgen.window(300, 300, 6, 0.7, seed=5, mode=0))
+    out.append(matgen.window(257, 500, 16, 0.9, seed=6, mode=1))
+    lens = np.zeros(400, np.int64)
+    lens[[3, 4, 200, 201, 202, 350]] = [1, 700, 5, 64, 1, 2000]
+    out.append(matgen.from_lengths(lens, 3000, seed=7))
+    out.append(matgen.rmat(9, seed=8))
+    out.append(matgen.from_lengths(np.random.default_rng(9).integers(0, 30, 123), 41, seed=9))
+    out.append(matgen.HostCSR(np.zeros(6, np.int64), np.zeros(0, np.int32), np.zeros(0), 5, 7))
+    out.append(matgen.from_lengths([1500], 1500, seed=10))              # one dense row
+    out.append(matgen.from_lengths(np.ones(700, np.int64), 1, seed=11))  # n x 1
+    return out
+
+
+N_CASES = 10
+
+
+# ------------------------------------------------------------------ COO / ELL / HYB
+
+def test_golden_coo_ell_hyb():
+    g = load("app_a_4x4.json")
+    A = csr_of(g)
+    assert oracle.csr2coo(A).tolist() == g["coo_row"]
+    e = oracle.csr2ell(A)
+    assert e["K"] == g["ell_K"] and e["ld"] == 32
+    for j in range(e["K"]):
+        assert e["col"][j * 32:j * 32 + 4].tolist() == g["ell_first4_by_slice"]["col"][j]
+        assert e["val"][j * 32:j * 32 + 4].tolist() == g["ell_first4_by_slice"]["val"][j]
+        assert np.all(e["col"][j * 32 + 4:(j + 1) * 32] == -1)
+    h = oracle.csr2hyb(A)
+    assert h["K"] == g["hyb"]["K"]
+    assert h["coo_row"].tolist() == g["hyb"]["coo_row"]
+    assert h["coo_col"].tolist() == g["hyb"]["coo_col"]
+    assert h["coo_val"].tolist() == g["hyb"]["coo_val"]
+    assert oracle.hyb_width(A, "floor") == g["hyb"]["K_floor"]
+    assert oracle.hyb_width(A, "cusp") == g["hyb"]["K_cusp"]
+
+
+@pytest.mark.parametrize("i", range(N_CASES))
+def test_ell_hyb_coo_round_trip(i):
+    """Decoding each format back to CSR gives the input (numpy decoders)."""
+    A = structured_cases()[i]
+    n = A.n_rows
+    lens = np.diff(A.row_ptr)
+    # COO
+    row = oracle.csr2coo(A)
+    assert np.array_equal(row, np.repeat(np.arange(n), lens))
+    # ELL: column-major slices; per-row the first len entries, then sentinels
+    e = oracle.csr2ell(A)
+    K, ld = e["K"], e["ld"]
+    assert K == (lens.max() if n else 0) and ld % 32 == 0 and ld >= n
+    C = e["col"].reshape(K, ld).T if K else np.zeros((ld, 0), np.int32)
+    V = e["val"].reshape(K, ld).T if K else np.zeros((ld, 0))
+    for r in range(n):
+        s, t = A.row_ptr[r], A.row_ptr[r + 1]
+        assert np.array_equal(C[r, :t - s], A.col[s:t]) and np.array_equal(V[r, :t - s], A.val[s:t])
+        assert np.all(C[r, t - s:] == -1) and np.all(V[r, t - s:] == 0)
+    assert np.all(C[n:] == -1)
+    # HYB
+    for rule in ("ceil", "floor", "cusp"):
+        h = oracle.csr2hyb(A, rule)
+        Kh = h["K"]
+        HC = h["ell_col"].reshape(Kh, ld).T if Kh else np.zeros((ld, 0), np.int32)
+        rows_c, cols_c, vals_c = [], [], []
+        for r in range(n):
+            s, t = A.row_ptr[r], A.row_ptr[r + 1]
+            m = min(t - s, Kh)
+            assert np.array_equal(HC[r, :m], A.col[s:s + m]) and np.all(HC[r, m:] == -1)
+            rows_c += [r] * (t - s - m)
+            cols_c += A.col[s + m:t].tolist()
+            vals_c += A.val[s + m:t].tolist()
+        assert h["coo_row"].tolist() == rows_c and h["coo_col"].tolist() == cols_c
+        assert h["coo_val"].tolist() == vals_c
+
+
+def test_hyb_width_rules_definitions():
+    """A2: ceil/floor of nnz_mu; the [2]-style rule by brute definition over k."""
+    for A in structured_cases():
+        n = A.n_rows
+        lens = np.diff(A.row_ptr)
+        nnz = A.nnz
+        assert oracle.hyb_width(A, "ceil") == (-(-nnz // n) if n else 0)
+        assert oracle.hyb_width(A, "floor") == (nnz // n if n else 0)
+        K = int(lens.max()) if n else 0
+        exp = K
+        for k in range(K):
+            longer = int((lens > k).sum())
+            if 3 * longer < n or longer < 4096:
+                exp = k
+                break
+        assert oracle.hyb_width(A, "cusp") == (exp if n else 0)
+
+
+# ------------------------------------------------------------------ merge path
+
+def merge_coord_formula(row_ptr, d):
+    """A7 closed form: i = largest i in [0, min(d, n)] with row_ptr[i] + i <= d."""
+    n = row_ptr.size - 1
+    key = row_ptr + np.arange(n + 1)
+    i = int(np.searchsorted(key, d, side="right")) - 1
+    i = min(i, min(d, n))
+    return i, d - i
+
+
+@pytest.mark.parametrize("name", ["app_a_4x4.json", "app_a_5x5.json"])
+def test_golden_merge_coords(name):
+    g = load(name)
+    A = csr_of(g)
+    cr, cn = oracle.merge_coords(A, 1)
+    assert [[int(a), int(b)] for a, b in zip(cr, cn)] == g["merge_coords_T1"]
+
+
+@pytest.mark.parametrize("T", [1, 3, 7, 64, 1000])
+def test_merge_walk_equals_binary_search(T):
+    for A in structured_cases():
+        cr, cn = oracle.merge_coords(A, T)
+        total = A.n_rows + A.nnz
+        nt = -(-total // T)
+        assert cr.size == nt + 1
+        for t in range(nt + 1):
+            d = min(t * T, total)
+            assert (cr[t], cn[t]) == merge_coord_formula(A.row_ptr, d)
+        assert cr[-1] == A.n_rows and cn[-1] == A.nnz
+        assert np.all(np.diff(cr) >= 0) and np.all(np.diff(cn) >= 0)
+
+
+# ------------------------------------------------------------------ partition
+
+@pytest.mark.parametrize("name", ["app_a_4x4.json", "app_a_5x5.json"])
+def test_golden_partition(name):
+    g = load(name)
+    A = csr_of(g)
+    for P, exp in g["partition"].items():
+        assert oracle.partition(A, int(P)).tolist() == exp
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
+def test_partition_invariants(P):
+    for A in structured_cases():
+        s = oracle.partition(A, P)
+        total = A.n_rows + A.nnz
+        assert s[0] == 0 and s[-1] == A.n_rows and np.all(np.diff(s) >= 0)
+        lens = np.diff(A.row_ptr)
+        longest = int(lens.max()) if A.n_rows else 0
+        for k in range(P):
+            assert s[k] == merge_coord_formula(A.row_ptr, (k * total) // P)[0]
+            items = (s[k + 1] - s[k]) + (A.row_ptr[s[k + 1]] - A.row_ptr[s[k]])
+            assert items <= -(-total // P) + longest + 1
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 5])
+def test_slice_remap_reassembles_spmv(P):
+    """Shard SpMV with the gathered (padded) x equals the unpartitioned oracle bit-exactly."""
+    A = matgen.rmat(10, seed=21)
+    x = matgen.vector(A.n_cols, 21, 1)
+    y = matgen.vector(A.n_rows, 21, 2)
+    s = oracle.partition(A, P)
+    S = oracle.partition_slot(s)
+    xg = np.zeros(P * S)
+    for k in range(P):
+        xg[k * S:k * S + s[k + 1] - s[k]] = x[s[k]:s[k + 1]]
+    full = oracle.spmv_csr(A, x, 1.5, -0.5, y)
+    for k in range(P):
+        rp, col, val = oracle.slice_remap(A, s, k)
+        shard = matgen.HostCSR(rp, col, val, int(s[k + 1] - s[k]), P * S)
+        part = oracle.spmv_csr(shard, xg, 1.5, -0.5, y[s[k]:s[k + 1]])
+        assert np.array_equal(part, full[s[k]:s[k + 1]])
+
+
+# ------------------------------------------------------------------ CSR5
+
+def test_csr5_sigma_rule():
+    """A6: sigma = clamp(4*ceil(ceil(nnz_mu)/4), 4, 16)."""
+    assert oracle.csr5_sigma(matgen.laplacian5(16)) == 8          # mu ~ 4.7 -> 5 -> 8
+    assert oracle.csr5_sigma(matgen.uniform_fixed(64, 64, 16)) == 16
+    assert oracle.csr5_sigma(matgen.uniform_fixed(64, 64, 1)) == 4
+    assert oracle.csr5_sigma(matgen.uniform_fixed(64, 64, 40)) == 16
+
+
+@pytest.mark.parametrize("i", range(N_CASES))
+@pytest.mark.parametrize("val_bytes", [4, 8])
+@pytest.mark.parametrize("sigma", [None, 4, 16])
+def test_csr5_round_trip_and_invariants(i, val_bytes, sigma):
+    A = structured_cases()[i]
+    e = oracle.csr5_encode(A, val_bytes=val_bytes, sigma=sigma)
+    sg = e["sigma"]
+    W = 32 * sg
+    nt = e["n_tiles"]
+    assert nt == A.nnz // W
+    rc, rp, col, val = oracle.csr5_decode((A.n_rows, A.nnz), e, A.row_ptr, val_bytes)
+    assert rc == 0
+    assert np.array_equal(rp, A.row_ptr) and np.array_equal(col, A.col) and np.array_equal(val, A.val)
+    # invariants: popcounts = non-empty rows starting inside full tiles
+    desc = e["tile_desc"].reshape(nt, 32) if nt else np.zeros((0, 32), np.uint32)
+    flags = desc & 0xFFFF
+    starts = A.row_ptr[:-1][np.diff(A.row_ptr) > 0]
+    assert sum(bin(int(f)).count("1") for f in flags.ravel()) == int((starts < nt * W).sum())
+    for t in range(nt):
+        yoff = (desc[t] >> 16) & 0x1FF
+        pc = np.array([bin(int(f)).count("1") for f in flags[t]])
+        assert np.array_equal(yoff, np.concatenate([[0], np.cumsum(pc)[:-1]]))
+        for l in range(32):
+            m = 0
+            while l + m + 1 < 32 and flags[t, l + m + 1] == 0:
+                m += 1
+            assert (desc[t, l] >> 25) & 0x1F == m
+    assert np.all(np.diff(e["row_lo"]) >= 0)
+    # row_lo[t] = first row whose start >= t*W (A6)
+    for t in range(nt + 1):
+        exp = int(np.searchsorted(A.row_ptr[:-1], t * W, side="left"))
+        assert e["row_lo"][t] == exp
+
+
+def test_csr5_decode_detects_corruption():
+    A = matgen.rmat(9, seed=8)
+    e = oracle.csr5_encode(A)
+    assert e["n_tiles"] > 2
+    bad = dict(e)
+    bad["tile_desc"] = e["tile_desc"].copy()
+    bad["tile_desc"][33] ^= (1 << 16)          # y_offset off by one
+    assert oracle.csr5_decode((A.n_rows, A.nnz), bad, A.row_ptr)[0] != 0
+    bad2 = dict(e)
+    bad2["tile_ptr"] = e["tile_ptr"].copy()
+    bad2["tile_ptr"][1] += 1
+    assert oracle.csr5_decode((A.n_rows, A.nnz), bad2, A.row_ptr)[0] != 0
+
+
+def test_csr5_layout_is_lane_interleaved():
+    """A6 layout: element e = t*W + l*sigma + s at t*W + (s//v)*32*v + l*v + s%v."""
+    A = matgen.uniform_fixed(256, 4096, 16, seed=3)
+    e = oracle.csr5_encode(A, val_bytes=8)
+    sg, W = e["sigma"], 32 * e["sigma"]
+    for (t, l, s) in [(0, 0, 0), (0, 5, 3), (1, 31, 15), (2, 7, 9)]:
+        src = t * W + l * sg + s
+        assert e["col_perm"][t * W + (s // 4) * 128 + l * 4 + s % 4] == A.col[src]
+        assert e["val_perm"][t * W + (s // 2) * 64 + l * 2 + s % 2] == A.val[src]
+
+
+# ------------------------------------------------------------------ features
+
+def features_brute(A):
+    """numpy/python brute force of Table II per A8/A9 (independent of oracle.c)."""
+    n, m = A.n_rows, A.n_cols
+    lens = np.diff(A.row_ptr).astype(np.int64)
+    blocks, bsizes = [], []
+    for r in range(n):
+        c = A.col[A.row_ptr[r]:A.row_ptr[r + 1]].astype(np.int64)
+        if c.size == 0:
+            blocks.append(0)
+            continue
+        cuts = np.nonzero(np.diff(c) != 1)[0]
+        edges = np.concatenate([[0], cuts + 1, [c.size]])
+        sizes = np.diff(edges)
+        blocks.append(sizes.size)
+        bsizes += sizes.tolist()
+    blocks = np.array(blocks, np.int64)
+    bs = np.array(bsizes, np.int64)
+    nnz = int(lens.sum())
+
+    def sig(vals, cnt):
+        S1, S2 = int(vals.sum()), int((vals.astype(object) ** 2).sum()) if vals.size else 0
+        return float(np.sqrt(float(cnt * S2 - S1 * S1))) / cnt if cnt else 0.0
+
+    f = dict(n_rows=n, n_cols=m, nnz_tot=nnz,
+             nnz_mu=nnz / n if n else 0.0,
+             nnz_frac=float(100 * nnz) / float(n * m) if n and m else 0.0,
+             nnz_max=int(lens.max()) if n else 0, nnz_min=int(lens.min()) if n else 0,
+             nnz_sigma=sig(lens, n),
+             nnzb_tot=int(blocks.sum()), nnzb_mu=float(blocks.sum()) / n if n else 0.0,
+             nnzb_sigma=sig(blocks, n),
+             nnzb_min=int(blocks.min()) if n else 0, nnzb_max=int(blocks.max()) if n else 0,
+             snzb_mu=nnz / bs.size if bs.size else 0.0, snzb_sigma=sig(bs, bs.size),
+             snzb_min=int(bs.min()) if bs.size else 0, snzb_max=int(bs.max()) if bs.size else 0,
+             n_empty_rows=int((lens == 0).sum()))
+    f["ell_width"] = f["nnz_max"]
+    f["ell_slots"] = f["nnz_max"] * n
+    f["ell_pad_frac"] = (f["ell_slots"] - nnz) / f["ell_slots"] if f["ell_slots"] else 0.0
+    return f
+
+
+@pytest.mark.parametrize("name", ["app_a_4x4.json", "app_a_5x5.json"])
+def test_golden_features(name):
+    g = load(name)
+    f = oracle.features(csr_of(g))
+    for k, v in g["features"].items():
+        assert f[k] == v, k
+
+
+@pytest.mark.parametrize("i", range(N_CASES))
+def test_features_vs_brute_force(i):
+    A = structured_cases()[i]
+    f = oracle.features(A)
+    for k, v in features_brute(A).items():
+        assert f[k] == v, (k, f[k], v)
+
+
+def test_features_lap4096_closed_forms():
+    """App. B closed forms with m = g - 2, evaluated here from the formulas."""
+    g = load("app_b_lap4096.json")
+    G = g["g"]
+    m = G - 2
+    A = matgen.laplacian5(G)
+    f = oracle.features(A)
+    assert f["nnz_tot"] == 5 * G * G - 4 * G
+    assert f["sum_len2"] == 25 * m * m + 64 * m + 36
+    assert f["nnzb_tot"] == 3 * m * m + 10 * m + 8
+    assert f["sum_nnzb2"] == 9 * m * m + 26 * m + 16
+    assert f["sum_snzb2"] == 11 * m * m + 32 * m + 20
+    for k, v in g["features"].items():
+        assert f[k] == v, k
+    assert f["ell_pad_frac"] == 1 / 5120
+
+
+@pytest.mark.parametrize("G", [3, 4, 5, 8])
+def test_features_laplacian_small_brute(G):
+    A = matgen.laplacian5(G)
+    f = oracle.features(A)
+    for k, v in features_brute(A).items():
+        assert f[k] == v, k
+
+
+def test_features_u2048():
+    """cfg1 closed forms: 16 per row, nnz_frac 0.78125, pad 0, K_h 16, K_cusp 0."""
+    A = matgen.uniform_fixed(2048, 2048, 16)
+    f = oracle.features(A)
+    assert f["nnz_max"] == f["nnz_min"] == 16 and f["nnz_sigma"] == 0.0
+    assert f["nnz_frac"] == 0.78125 and f["ell_pad_frac"] == 0.0
+    assert f["hyb_width"] == 16 and f["hyb_width_cusp"] == 0
