@@ -1,0 +1,255 @@
+/*
+ * spmv.h -- C ABI of libspmv: six-format SpMV y <- alpha*A*x + beta*y, the
+ * CSR -> format converters, per-matrix sparsity features and the multi-GPU row
+ * partition, hand-written for B200 (sm_100a).
+ *
+ * Paper: Nisa, Siegel, Sukumaran Rajam, Vishnu, Sadayappan, "Effective Machine
+ * Learning Based Format Selection and Performance Modeling for SpMV on GPUs",
+ * IPDPSW 2018.  PAPER.md:<n> = line n of the text extraction; A<n> = reading n of
+ * the ambiguity register (restated in DESIGN.md §3).
+ *
+ * General rules
+ *  - Plain C types only.  "device" pointers are CUDA device memory on the ctx's
+ *    device; "host" pointers are ordinary host memory.
+ *  - Every call returns an spmv_status; nothing aborts and no C++ exception crosses
+ *    the ABI.  On error, spmv_last_error() returns a thread-local detail string.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *    All device work is stream-ordered on it.
+ *  - Inputs are BORROWED for the duration of the call (stream-ordered) and never
+ *    retained, unless stated.  A handle OWNS every device array it allocates.
+ *  - No CPU fallback exists: without a usable sm_100 device every entry point
+ *    that would touch the device returns SPMV_ERR_UNSUPPORTED or SPMV_ERR_CUDA.
+ */
+#ifndef SPMV_H
+#define SPMV_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* exported symbols stay visible when the library is built with -fvisibility=hidden */
+#if defined(__GNUC__)
+#pragma GCC visibility push(default)
+#endif
+
+#define SPMV_ABI_VERSION 1
+
+typedef enum {
+    SPMV_OK = 0,
+    SPMV_ERR_INVALID_ARG = 1,   /* null/inconsistent argument, x/y overlap, bad id   */
+    SPMV_ERR_NOT_CANONICAL = 2, /* row_ptr not monotone / not [0..nnz], column out of
+                                   range, unsorted or duplicate column in a row (A15) */
+    SPMV_ERR_SIZE = 3,          /* ELL/HYB slots exceed the size guard (A4), or an
+                                   index does not fit its type                        */
+    SPMV_ERR_NO_MEMORY = 4,     /* allocator returned NULL                            */
+    SPMV_ERR_CUDA = 5,          /* a CUDA runtime call or kernel launch failed        */
+    SPMV_ERR_UNSUPPORTED = 6    /* device is not sm_100, or dtype/format mismatch     */
+} spmv_status;
+
+/* The six formats of the study, in the paper's Fig. 3 order,
+ * plus the CSR-scalar kernel variant (a variant, not a label, A5). */
+typedef enum {
+    SPMV_COO = 0,        /* PAPER.md:89  (§II-A.1) */
+    SPMV_ELL = 1,        /* PAPER.md:93  (§II-A.3) */
+    SPMV_CSR = 2,        /* PAPER.md:91  (§II-A.2), CSR-vector kernel (A5) */
+    SPMV_HYB = 3,        /* PAPER.md:95  (§II-A.4) */
+    SPMV_MERGE = 4,      /* PAPER.md:103 (§II-A.6) */
+    SPMV_CSR5 = 5,       /* PAPER.md:97-101 (§II-A.5) */
+    SPMV_CSR_SCALAR = 6  /* PAPER.md:91, one thread per row */
+} spmv_format;
+
+typedef enum { SPMV_F32 = 0, SPMV_F64 = 1 } spmv_dtype;   /* value type (fp32 accumulates in fp64, A13) */
+typedef enum { SPMV_I32 = 0, SPMV_I64 = 1 } spmv_itype;   /* row_ptr type (A17) */
+
+/* Canonical CSR matrix, all pointers DEVICE, borrowed.
+ * row_ptr[n_rows+1] (ptr_type), col_idx[nnz] int32, vals[nnz] (dtype).
+ * Canonical = row_ptr[0]=0, monotone, row_ptr[n_rows]=nnz, columns strictly
+ * increasing within a row and in [0, n_cols) (A15). */
+typedef struct {
+    int64_t n_rows, n_cols, nnz;
+    spmv_itype ptr_type;
+    const void *row_ptr;
+    const int32_t *col_idx;
+    const void *vals;
+    spmv_dtype dtype;
+} spmv_csr;
+
+/* Device allocator used for every allocation of a ctx (handles, scratch).
+ * alloc(bytes, device, stream, user) returns a device pointer or NULL;
+ * free(ptr, bytes, device, stream, user) is stream-ordered.
+ * NULL allocator in spmv_init => cudaMallocAsync / cudaFreeAsync. */
+typedef struct {
+    void *(*alloc)(size_t bytes, int device, void *stream, void *user);
+    void (*free)(void *ptr, size_t bytes, int device, void *stream, void *user);
+    void *user;
+} spmv_allocator;
+
+typedef struct spmv_ctx spmv_ctx;
+typedef struct spmv_handle spmv_handle;
+
+/* ---- context ------------------------------------------------------------- */
+
+/* Bind to `device` (must be compute capability 10.0, else SPMV_ERR_UNSUPPORTED).
+ * The allocator struct is copied.  *out receives a ctx owned by the caller. */
+spmv_status spmv_init(int device, const spmv_allocator *alloc, spmv_ctx **out);
+/* Release the ctx (handles created from it must be destroyed first). */
+spmv_status spmv_finalize(spmv_ctx *ctx);
+/* Device SM count and L2 size the library sized its grids for (host outputs). */
+spmv_status spmv_device_info(const spmv_ctx *ctx, int *sm_count, int64_t *l2_bytes);
+
+/* ---- features (Table II; §IV-A) ---------- */
+
+/* The 17 features of the paper under the names of its Figs 4-5,
+ * read per A8 (nnz_frac in percent, population sigma, a block = maximal run of
+ * consecutive columns within a row, nnzb_* over all rows, snzb_* over all blocks),
+ * computed from exact integer sums by the fixed fp64 formulas of A9; plus the
+ * north_star extras (ELL padding ratio, HYB split widths). */
+typedef struct {
+    int64_t n_rows, n_cols, nnz_tot;
+    double nnz_mu, nnz_frac;
+    int64_t nnz_max;  double nnz_sigma;
+    double nnzb_mu, nnzb_sigma, snzb_mu, snzb_sigma;
+    int64_t nnzb_tot, nnzb_min, nnzb_max, snzb_min, snzb_max, nnz_min;
+    int64_t ell_width, ell_slots;  double ell_pad_frac;
+    int64_t hyb_width, hyb_coo_nnz, hyb_width_floor, hyb_width_cusp;  /* PAPER.md:95, A2 */
+    int64_t n_empty_rows;
+    uint64_t sum_len2, sum_nnzb2, sum_snzb2;              /* exact sums behind the sigmas */
+} spmv_features_t;
+
+/* One O(nnz) device pass over row_ptr + col_idx (vals are not read), then one
+ * device->host readback: BLOCKS on `stream`.  Returns SPMV_ERR_NOT_CANONICAL
+ * for a non-canonical matrix (out_host is then unspecified). */
+spmv_status spmv_features(spmv_ctx *ctx, const spmv_csr *A, void *stream,
+                          spmv_features_t *out_host);
+
+/* ---- conversion ------------------------------------------------------------ */
+
+typedef struct {
+    int hyb_rule;          /* 0 = ceil(nnz/n_rows) (default; "nnz_mu, which we
+                              use", A2), 1 = floor, 2 = the max(4096, rows/3)-style rule   */
+    int64_t hyb_width;     /* >= 0 overrides hyb_rule; < 0 = use the rule                 */
+    int csr5_sigma;        /* 0 = A6 rule clamp(4*ceil(ceil(nnz_mu)/4), 4, 16); else 4..16, %4 */
+    int merge_items;       /* merge-path items per CTA (0 = default); recorded in info     */
+    int vector_width;      /* CSR-vector lanes per row (0 = A5 rule), power of two 1..32  */
+    size_t max_bytes;      /* ELL/HYB guard (0 = min(1/2 free memory, max(8x the CSR bytes,
+                              64 MiB)))                                                    */
+    int alias_input;       /* 1 = COO/CSR/MERGE handles reference the caller's col/vals
+                              (caller keeps them alive and unchanged)                     */
+} spmv_convert_opts;
+
+/* Fill `opts` with the defaults (all rules as above). */
+void spmv_convert_opts_default(spmv_convert_opts *opts);
+
+/* Build a handle holding A in format `fmt` (CSR -> COO/ELL/HYB/merge-partition/
+ * CSR5-tile descriptors, layouts DESIGN.md §4).  Validates A (the
+ * feature pass's canonical check), does one blocking size readback, checks the size
+ * guard (ELL/HYB: SPMV_ERR_SIZE, A4), allocates through the ctx allocator on
+ * `stream`, launches the conversion on `stream` and returns.  opts may be NULL. */
+spmv_status spmv_convert(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A,
+                         const spmv_convert_opts *opts, void *stream, spmv_handle **out);
+
+/* y <- alpha*A*x + beta*y (BLAS conventions, A14): beta == 0 => y is write-only;
+ * alpha == 0 => A is not read.  alpha/beta are HOST scalars of the handle's dtype
+ * (float* or double*), copied at call time.  x (n_cols) and y (n_rows) are DEVICE
+ * arrays of the handle's dtype; they must not overlap (SPMV_ERR_INVALID_ARG).
+ * Fully asynchronous on `stream` (CUDA-graph capturable); a handle runs on one
+ * stream at a time (it owns per-run carry scratch).  Summation is deterministic:
+ * fixed-order segmented sums, no floating-point atomics. */
+spmv_status spmv_run(spmv_handle *h, const void *alpha, const void *x,
+                     const void *beta, void *y, void *stream);
+
+/* End-to-end variant for HOST x/y (pageable or pinned): copies x (and y when
+ * beta != 0) host->device into handle-owned buffers, runs, copies y back, and
+ * synchronizes `stream` before returning. */
+spmv_status spmv_run_host(spmv_handle *h, const void *alpha, const void *x_host,
+                          const void *beta, void *y_host, void *stream);
+
+/* Number of kernel launches one spmv_run issues for this handle (host output). */
+spmv_status spmv_run_launches(const spmv_handle *h, int *launches);
+
+typedef struct {
+    spmv_format format;
+    spmv_dtype dtype;
+    spmv_itype ptr_type;            /* index type used inside the handle */
+    int64_t n_rows, n_cols, nnz;
+    int64_t ell_width, ell_ld;      /* ELL / HYB-ELL part */
+    int64_t hyb_coo_nnz;            /* HYB COO part */
+    int64_t csr5_sigma, csr5_tiles, csr5_map_len;
+    int64_t merge_items, merge_tiles;
+    int64_t vector_width;
+    size_t device_bytes;            /* bytes owned by the handle */
+    size_t bytes_per_run;           /* algorithmic bytes of one run with beta != 0
+                                       (format's own storage + x + y read + y write),
+                                       DESIGN.md §6 */
+    size_t bytes_per_run_beta0;     /* same with beta == 0 (y not read) */
+} spmv_handle_info;
+
+spmv_status spmv_info(const spmv_handle *h, spmv_handle_info *out_host);
+
+/* Arrays a handle can export for bit-exact tests (layouts: DESIGN.md §4). */
+typedef enum {
+    SPMV_ARR_ROW_PTR = 0,    /* CSR/MERGE/CSR5/CSR_SCALAR row_ptr (ptr_type)          */
+    SPMV_ARR_COL = 1,        /* CSR/MERGE/COO col (int32); CSR5: lane-interleaved col */
+    SPMV_ARR_VAL = 2,        /* as above, values (dtype)                               */
+    SPMV_ARR_COO_ROW = 3,    /* COO / HYB-COO row (int32)                              */
+    SPMV_ARR_ELL_COL = 4,    /* ELL / HYB-ELL, K*ld int32, col = -1 padding            */
+    SPMV_ARR_ELL_VAL = 5,    /* ELL / HYB-ELL, K*ld dtype, +0.0 padding                */
+    SPMV_ARR_HYB_COO_COL = 6,
+    SPMV_ARR_HYB_COO_VAL = 7,
+    SPMV_ARR_MERGE_COORD_ROW = 8,   /* int64 [tiles+1] */
+    SPMV_ARR_MERGE_COORD_NZ = 9,    /* int64 [tiles+1] */
+    SPMV_ARR_CSR5_TILE_PTR = 10,    /* int64 [tiles+1] */
+    SPMV_ARR_CSR5_ROW_LO = 11,      /* int64 [tiles+1] */
+    SPMV_ARR_CSR5_TILE_DESC = 12,   /* uint32 [tiles*32] */
+    SPMV_ARR_CSR5_MAP_OFF = 13,     /* int64 [tiles] (-1 = no empty row in range) */
+    SPMV_ARR_CSR5_SEG_MAP = 14      /* int64 [map_len] */
+} spmv_array_id;
+
+/* Copy array `id` of the handle to host memory (blocking on `stream`).
+ * *written = bytes of the array; SPMV_ERR_INVALID_ARG if the handle has no such
+ * array or cap < size (then *written still reports the size). */
+spmv_status spmv_export(const spmv_handle *h, spmv_array_id id, void *host_dst,
+                        size_t cap, size_t *written, void *stream);
+
+/* Free the handle's arrays (stream-ordered on `stream`) and the handle. */
+spmv_status spmv_destroy(spmv_handle *h, void *stream);
+
+/* ---- multi-GPU row partition (north_star) --------------------- */
+
+/* nnz-balanced merge-path row splits: splits[k] = row coordinate of the merge path
+ * of A's row ends with its nonzeros at diagonal floor(k*(n_rows+nnz)/nparts),
+ * k = 0..nparts (row-aligned; a straddling row goes to the later part).
+ * row_splits_host[nparts+1] is HOST output.  Blocks on `stream`. */
+spmv_status spmv_partition(spmv_ctx *ctx, const spmv_csr *A, int nparts, void *stream,
+                           int64_t *row_splits_host);
+
+/* Size of shard `part`: rows = splits[part+1]-splits[part], nnz of those rows and the
+ * gathered-x slot size S = max part rows (all host outputs; blocks on `stream`). */
+spmv_status spmv_slice_size(spmv_ctx *ctx, const spmv_csr *A, const int64_t *row_splits_host,
+                            int nparts, int part, void *stream,
+                            int64_t *rows, int64_t *nnz, int64_t *slot);
+
+/* Shard `part` of a SQUARE matrix into caller-allocated DEVICE arrays:
+ * row_ptr_out[rows+1] int32 (rebased to 0; SPMV_ERR_SIZE if shard nnz > INT32_MAX),
+ * col_out[nnz] int32 remapped to the gathered-x slot owner(j)*S + (j - splits[owner]),
+ * vals_out[nnz] (A's dtype).  Asynchronous on `stream`. */
+spmv_status spmv_slice_remap(spmv_ctx *ctx, const spmv_csr *A, const int64_t *row_splits_host,
+                             int nparts, int part, void *stream,
+                             int32_t *row_ptr_out, int32_t *col_out, void *vals_out);
+
+/* ---- diagnostics ----------------------------------------------------------- */
+const char *spmv_status_str(spmv_status s);
+const char *spmv_last_error(void);
+int spmv_abi_version(void);
+
+#if defined(__GNUC__)
+#pragma GCC visibility pop
+#endif
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPMV_H */

@@ -1,0 +1,114 @@
+"""Per-format timing and best-format labels (§IV-B):
+
+    "The execution time is collected by executing each matrix multiple (50) times
+     and then averaging the execution time.  We label the format with minimum
+     execution time (maximum GFLOPS) as the best format."
+
+Readings: A10 GFLOP/s = 2*nnz/t with the true nnz; A11 5 warm-ups,
+one CUDA-event pair around 50 back-to-back runs -> mean (the label metric), per-call
+events -> median/min, hot L2, alpha = beta = 1; A12 label6 / label5 (no COO,
+PAPER.md:235) / label3 (ELL, CSR, HYB), exact ties to the paper's
+Fig. 3 order, margin = t_2nd/t_best - 1; A4 infeasible formats are
+"N/A" and excluded from the argmin.
+
+Timing only: no oracle here.  All device work runs in libspmv kernels.
+"""
+from __future__ import annotations
+
+import statistics
+from typing import Dict, Iterable, List, Optional
+
+import torch
+
+from .spmv import CSR, PAPER_FORMATS, SpmvError, convert
+
+LABEL_SETS = {
+    "label6": ("coo", "ell", "csr", "hyb", "merge", "csr5"),
+    "label5": ("ell", "csr", "hyb", "merge", "csr5"),
+    "label3": ("ell", "csr", "hyb"),
+}
+
+
+def time_handle(h, x: torch.Tensor, y: torch.Tensor, reps: int = 50, warmup: int = 5,
+                alpha: float = 1.0, beta: float = 1.0, per_call: bool = True) -> Dict[str, float]:
+    """A11 protocol on the current stream.  Returns mean (batch event pair), median and
+    min of per-call events, in milliseconds."""
+    s = torch.cuda.current_stream()
+    for _ in range(warmup):
+        h.run(alpha, x, beta, y)
+    s.synchronize()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t0.record(s)
+    for _ in range(reps):
+        h.run(alpha, x, beta, y)
+    t1.record(s)
+    s.synchronize()
+    out = {"t_mean_ms": t0.elapsed_time(t1) / reps, "reps": reps}
+    if per_call:
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+        for a, b in evs:
+            a.record(s)
+            h.run(alpha, x, beta, y)
+            b.record(s)
+        s.synchronize()
+        ts = [a.elapsed_time(b) for a, b in evs]
+        out["t_median_ms"] = statistics.median(ts)
+        out["t_min_ms"] = min(ts)
+    return out
+
+
+def labels(times_ms: Dict[str, Optional[float]]) -> Dict[str, object]:
+    """A12: argmin over feasible formats per label set; exact ties in Fig. 3 order."""
+    out: Dict[str, object] = {}
+    for name, fmts in LABEL_SETS.items():
+        feas = [(times_ms[f], PAPER_FORMATS.index(f), f) for f in fmts if times_ms.get(f) is not None]
+        if not feas:
+            out[name] = None
+            continue
+        feas.sort()
+        out[name] = feas[0][2]
+        if name == "label6":
+            out["margin"] = (feas[1][0] / feas[0][0] - 1.0) if len(feas) > 1 and feas[0][0] > 0 else None
+    return out
+
+
+def measure_matrix(A: CSR, formats: Iterable[str] = PAPER_FORMATS, reps: int = 50, warmup: int = 5,
+                   x: Optional[torch.Tensor] = None, y: Optional[torch.Tensor] = None,
+                   **convert_opts) -> Dict[str, object]:
+    """Convert A to each format, time it, and emit the per-format record + labels
+    (the paper's ground truth, regenerated on this GPU)."""
+    dev = A.row_ptr.device
+    if x is None:
+        x = torch.ones(A.n_cols, dtype=A.dtype, device=dev)
+    if y is None:
+        y = torch.zeros(A.n_rows, dtype=A.dtype, device=dev)
+    rec: Dict[str, object] = {"formats": {}}
+    times: Dict[str, Optional[float]] = {}
+    for f in formats:
+        try:
+            h = convert(A, f, **convert_opts)
+        except SpmvError as e:
+            if e.status in (3, 4):          # SPMV_ERR_SIZE / NO_MEMORY -> N/A (A4)
+                rec["formats"][f] = {"status": "N/A", "reason": e.name}
+                times[f] = None
+                continue
+            raise
+        t = time_handle(h, x, y, reps=reps, warmup=warmup)
+        info = h.info()
+        gflops = 2.0 * A.nnz / (t["t_mean_ms"] * 1e-3) / 1e9 if t["t_mean_ms"] > 0 else 0.0
+        gbs = info["bytes_per_run"] / (t["t_mean_ms"] * 1e-3) / 1e9 if t["t_mean_ms"] > 0 else 0.0
+        rec["formats"][f] = {**t, "gflops": gflops, "gbs_own": gbs, "bytes_per_run": info["bytes_per_run"],
+                             "launches": h.launches()}
+        times[f] = t["t_mean_ms"]
+        h.destroy()
+    rec.update(labels(times))
+    return rec
+
+
+def best_format(rec: Dict[str, object]) -> Optional[str]:
+    return rec.get("label6")  # type: ignore[return-value]
+
+
+def records_to_rows(recs: List[Dict[str, object]]) -> List[Dict[str, object]]:
+    """Flatten measure_matrix records (one JSONL line per matrix)."""
+    return [dict(r) for r in recs]

@@ -1,0 +1,419 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bars (north_star): conversions, partitions and integer features
+bit-exact; fp64 |y - y_ref| <= 1e-12 * bound, fp32 1e-5 * bound, with
+bound_i = |alpha| sum_j |a_ij||x_j| + |beta||y_i|; the integer-exact regime (P5)
+bit-exact in every format.
+"""
+import numpy as np
+import pytest
+import torch
+
+import matgen
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+ALPHA_BETA = [(1.0, 0.0), (1.5, -0.5), (0.0, 2.0), (-1.0, 1.0)]
+ALL_FORMATS = ("coo", "ell", "csr", "hyb", "merge", "csr5", "csr_scalar")
+TOL = {torch.float64: 1e-12, torch.float32: 1e-5}
+KIND = {torch.float64: "f64", torch.float32: "f32"}
+
+
+@pytest.fixture(scope="module")
+def sp():
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_nisassvs18_b200 as pkg
+    return pkg
+
+
+def _lens_matrix(lens, n_cols, seed, kind="f64"):
+    return matgen.from_lengths(np.asarray(lens, np.int64), n_cols, seed=seed, kind=kind)
+
+
+def edge_cases(kind="f64"):
+    """Edge suite of SURVEY §4 T2 (shapes, empty rows, long rows, tile boundaries)."""
+    rng = np.random.default_rng(1234)
+    cases = {}
+    cases["empty0x0"] = matgen.HostCSR(np.zeros(1, np.int64), np.zeros(0, np.int32), np.zeros(0), 0, 0)
+    cases["1x1"] = _lens_matrix([1], 1, 1, kind)
+    cases["dense_row_1x5000"] = _lens_matrix([5000], 5000, 2, kind)
+    cases["col_n_x_1"] = _lens_matrix(np.ones(3000, np.int64), 1, 3, kind)
+    cases["rect_3x7"] = _lens_matrix([2, 7, 0], 7, 4, kind)
+    cases["rect_7x3"] = _lens_matrix([1, 0, 3, 2, 0, 0, 1], 3, 5, kind)
+    cases["nnz0_rows5"] = matgen.HostCSR(np.zeros(6, np.int64), np.zeros(0, np.int32), np.zeros(0), 5, 9)
+    lens = rng.integers(0, 12, 5000)
+    lens[:37] = 0                      # leading empty rows
+    lens[-53:] = 0                     # trailing empty rows
+    lens[1000:1400] = 0                # a run of empty rows
+    cases["empty_runs"] = _lens_matrix(lens, 4000, 6, kind)
+    lens = rng.integers(1, 6, 20000)
+    lens[7777] = 100000                # one long row amid short ones
+    cases["long_row"] = _lens_matrix(lens, 200000, 7, kind)
+    # rows exactly at / around CSR5 tile (32*sigma) and merge/COO CTA (2048) boundaries
+    cases["tile_bounds"] = _lens_matrix([511, 512, 513, 2047, 2048, 2049, 1, 0, 4095, 4096, 4097] * 7, 9000, 8, kind)
+    cases["u2048"] = matgen.uniform_fixed(2048, 2048, 16, kind=kind)          # configs[0]
+    cases["lap37"] = matgen.laplacian5(37, kind=kind)
+    cases["lap64"] = matgen.laplacian5(64, kind=kind)
+    cases["rmat12"] = matgen.rmat(12, seed=12, kind=kind)
+    cases["rmat15"] = matgen.rmat(15, seed=15, kind=kind)
+    cases["banded"] = matgen.window(3000, 3000, 9, 0.6, seed=9, mode=0, kind=kind)
+    cases["blockdiag"] = matgen.window(2500, 4000, 64, 0.8, seed=10, mode=1, kind=kind)
+    cases["poisson_rect"] = _lens_matrix(rng.poisson(20, 4000), 1500, 11, kind)
+    zero = _lens_matrix(rng.integers(0, 9, 700), 700, 12, kind)
+    cases["all_zero_vals"] = matgen.HostCSR(zero.row_ptr, zero.col, np.zeros(zero.nnz), zero.n_rows, zero.n_cols)
+    return cases
+
+
+_CASES = {}
+
+
+def case(name, kind):
+    if kind not in _CASES:
+        _CASES[kind] = edge_cases(kind)
+    return _CASES[kind][name]
+
+
+CASE_NAMES = ["empty0x0", "1x1", "dense_row_1x5000", "col_n_x_1", "rect_3x7", "rect_7x3", "nnz0_rows5",
+              "empty_runs", "long_row", "tile_bounds", "u2048", "lap37", "lap64", "rmat12", "rmat15",
+              "banded", "blockdiag", "poisson_rect", "all_zero_vals"]
+
+
+def _guard(A, V):
+    """spmv.h: default guard max(8x the CSR bytes, 64 MiB) (free memory is not binding here)."""
+    return max(8 * (A.nnz * (4 + V) + (A.n_rows + 1) * 4), 64 << 20)
+
+
+def ell_expected_infeasible(A, dtype):
+    K, ld = oracle.ell_dims(A)
+    V = 8 if dtype == torch.float64 else 4
+    return K * ld * (4 + V) > _guard(A, V)
+
+
+def hyb_expected_infeasible(A, dtype, rule="ceil"):
+    Kh = oracle.hyb_width(A, rule)
+    ld = oracle.ell_dims(A)[1]
+    V = 8 if dtype == torch.float64 else 4
+    ncoo = oracle.lib().ora_hyb_coo_nnz(A.n_rows, A.row_ptr.ctypes.data, Kh)
+    return Kh * ld * (4 + V) + ncoo * (8 + V) > _guard(A, V)
+
+
+def expected_infeasible(A, fmt, dtype):
+    return ((fmt == "ell" and ell_expected_infeasible(A, dtype)) or
+            (fmt == "hyb" and hyb_expected_infeasible(A, dtype)))
+
+
+def to_dev(sp, A, dtype):
+    return sp.CSR.from_host(A, dtype=dtype)
+
+
+def run_format(sp, A, dA, fmt, dtype, alpha, beta, x, y0, **opts):
+    h = sp.convert(dA, fmt, **opts)
+    xd = torch.from_numpy(x).cuda().to(dtype)
+    if beta == 0.0:
+        yd = torch.full((A.n_rows,), float("nan"), dtype=dtype, device="cuda")   # must not be read
+    else:
+        yd = torch.from_numpy(y0).cuda().to(dtype)
+    h.run(alpha, xd, beta, yd)
+    torch.cuda.synchronize()
+    out = yd.cpu().double().numpy()
+    return h, out
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32], ids=["f64", "f32"])
+@pytest.mark.parametrize("fmt", ALL_FORMATS)
+@pytest.mark.parametrize("name", CASE_NAMES)
+def test_spmv_parity(sp, name, fmt, dtype):
+    A = case(name, KIND[dtype])
+    dA = to_dev(sp, A, dtype)
+    x = matgen.vector(A.n_cols, 77, 1, KIND[dtype])
+    y0 = matgen.vector(A.n_rows, 77, 2, KIND[dtype])
+    if expected_infeasible(A, fmt, dtype):
+        with pytest.raises(sp.SpmvError) as e:
+            sp.convert(dA, fmt)
+        assert e.value.status == 3
+        return
+    for alpha, beta in ALPHA_BETA:
+        ref, bound = oracle.spmv_csr(A, x, alpha, beta, y0, with_bound=True)
+        h, out = run_format(sp, A, dA, fmt, dtype, alpha, beta, x, y0)
+        ok, ratio, nbad = oracle.check_tolerance(out, ref, bound, TOL[dtype])
+        assert ok, f"{name}/{fmt}/{dtype} a={alpha} b={beta}: {nbad} bad rows, max ratio {ratio}"
+        h.destroy()
+
+
+INT_CASES = ["rmat15", "lap64", "long_row", "tile_bounds", "empty_runs", "u2048", "poisson_rect", "dense_row_1x5000"]
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32], ids=["f64", "f32"])
+@pytest.mark.parametrize("fmt", ALL_FORMATS)
+@pytest.mark.parametrize("name", INT_CASES)
+def test_integer_regime_bit_exact(sp, name, fmt, dtype):
+    """P5: a, x in {+-1, +-2}, small integer y, integer alpha/beta: any summation order gives
+    the same bits, so every format must match the oracle exactly."""
+    base = case(name, "f64")
+    A = matgen.set_values(base, 991, "int")
+    dA = to_dev(sp, A, dtype)
+    if expected_infeasible(A, fmt, dtype):
+        pytest.skip("infeasible (A4)")
+    x = matgen.vector(A.n_cols, 5, 1, "int")
+    y0 = np.round(matgen.vector(A.n_rows, 5, 2, "f64") * 8)
+    for alpha, beta in [(1.0, 0.0), (2.0, -1.0), (-1.0, 2.0), (0.0, -2.0)]:
+        ref = oracle.spmv_csr(A, x, alpha, beta, y0)
+        h, out = run_format(sp, A, dA, fmt, dtype, alpha, beta, x, y0)
+        assert np.array_equal(out, ref), f"{name}/{fmt}: not bit-exact (alpha={alpha}, beta={beta})"
+        h.destroy()
+
+
+# ------------------------------------------------------------------ conversions
+
+CONV_CASES = ["u2048", "rmat12", "rmat15", "empty_runs", "tile_bounds", "lap64", "rect_7x3", "nnz0_rows5",
+              "long_row", "banded"]
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32], ids=["f64", "f32"])
+@pytest.mark.parametrize("name", CONV_CASES)
+def test_conversions_bit_exact(sp, name, dtype):
+    A = case(name, KIND[dtype])
+    dA = to_dev(sp, A, dtype)
+    npv = np.float64 if dtype == torch.float64 else np.float32
+    vb = 8 if dtype == torch.float64 else 4
+    # CSR copies the input
+    h = sp.convert(dA, "csr")
+    assert np.array_equal(h.export("row_ptr").astype(np.int64), A.row_ptr)
+    assert np.array_equal(h.export("col"), A.col)
+    assert np.array_equal(h.export("val"), A.val.astype(npv))
+    # COO
+    h = sp.convert(dA, "coo")
+    assert np.array_equal(h.export("coo_row"), oracle.csr2coo(A))
+    # ELL (A3)
+    if not ell_expected_infeasible(A, dtype):
+        h = sp.convert(dA, "ell")
+        e = oracle.csr2ell(A)
+        assert h.info()["ell_width"] == e["K"] and h.info()["ell_ld"] == e["ld"]
+        assert np.array_equal(h.export("ell_col"), e["col"])
+        assert np.array_equal(h.export("ell_val"), e["val"].astype(npv))
+    # HYB (A1/A2) with each width rule
+    for rule in ("ceil", "floor", "cusp"):
+        if hyb_expected_infeasible(A, dtype, rule):
+            continue
+        h = sp.convert(dA, "hyb", hyb_rule=rule)
+        e = oracle.csr2hyb(A, rule)
+        assert h.info()["ell_width"] == e["K"], rule
+        assert np.array_equal(h.export("ell_col"), e["ell_col"])
+        assert np.array_equal(h.export("ell_val"), e["ell_val"].astype(npv))
+        assert np.array_equal(h.export("coo_row"), e["coo_row"])
+        assert np.array_equal(h.export("hyb_coo_col"), e["coo_col"])
+        assert np.array_equal(h.export("hyb_coo_val"), e["coo_val"].astype(npv))
+    # merge-path coordinates (A7)
+    h = sp.convert(dA, "merge")
+    T = h.info()["merge_items"]
+    cr, cn = oracle.merge_coords(A, T)
+    assert np.array_equal(h.export("merge_coord_row"), cr)
+    assert np.array_equal(h.export("merge_coord_nz"), cn)
+    # CSR5 (A6), default sigma and each legal sigma
+    for sigma in (None, 4, 8, 12, 16):
+        h = sp.convert(dA, "csr5", csr5_sigma=sigma or 0)
+        e = oracle.csr5_encode(A, val_bytes=vb, sigma=sigma)
+        assert h.info()["csr5_sigma"] == e["sigma"]
+        assert np.array_equal(h.export("csr5_tile_ptr"), e["tile_ptr"])
+        assert np.array_equal(h.export("csr5_row_lo"), e["row_lo"])
+        assert np.array_equal(h.export("csr5_tile_desc"), e["tile_desc"])
+        assert np.array_equal(h.export("csr5_map_off"), e["map_off"])
+        assert np.array_equal(h.export("csr5_seg_map"), e["seg_map"])
+        assert np.array_equal(h.export("col"), e["col_perm"])
+        assert np.array_equal(h.export("val"), e["val_perm"].astype(npv))
+
+
+# ------------------------------------------------------------------ features
+
+@pytest.mark.parametrize("name", CASE_NAMES)
+def test_features_bit_exact(sp, name):
+    A = case(name, "f64")
+    f = sp.features(to_dev(sp, A, torch.float64))
+    fo = oracle.features(A)
+    for k, v in fo.items():
+        assert f[k] == v, (name, k, f[k], v)
+
+
+def test_features_lap4096_full_size(sp):
+    """configs[1] at full size: features equal the App. B closed forms via the oracle."""
+    A = matgen.laplacian5(4096)
+    f = sp.features(to_dev(sp, A, torch.float64))
+    fo = oracle.features(A)
+    for k, v in fo.items():
+        assert f[k] == v, k
+
+
+def test_int64_row_ptr_input(sp):
+    A = case("rmat12", "f64")
+    dA = sp.CSR.from_host(A, dtype=torch.float64, ptr_dtype=torch.int64)
+    f = sp.features(dA)
+    assert f["nnzb_tot"] == oracle.features(A)["nnzb_tot"]
+    x = matgen.vector(A.n_cols, 3, 1)
+    ref, bound = oracle.spmv_csr(A, x, 1.0, 0.0, None, with_bound=True)
+    for fmt in ("csr", "merge", "csr5", "coo"):
+        h, out = run_format(sp, A, dA, fmt, torch.float64, 1.0, 0.0, x, None)
+        assert oracle.check_tolerance(out, ref, bound, 1e-12)[0], fmt
+
+
+# ------------------------------------------------------------------ partition
+
+def square_cases():
+    rng = np.random.default_rng(99)
+    lens = rng.integers(0, 12, 5000)
+    lens[:37] = 0
+    lens[1000:1400] = 0
+    lens[-53:] = 0
+    out = {"empty_runs_sq": _lens_matrix(lens, 5000, 21)}
+    lens = rng.integers(1, 6, 20000)
+    lens[7777] = 15000
+    out["long_row_sq"] = _lens_matrix(lens, 20000, 22)
+    return out
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
+@pytest.mark.parametrize("name", ["rmat15", "empty_runs_sq", "lap64", "long_row_sq", "u2048", "banded"])
+def test_partition_and_remap_bit_exact(sp, name, P):
+    """Remap needs a square matrix (x is owned in the row ranges of y)."""
+    A = square_cases()[name] if name.endswith("_sq") else case(name, "f64")
+    dA = to_dev(sp, A, torch.float64)
+    splits = sp.partition(dA, P)
+    assert np.array_equal(splits, oracle.partition(A, P))
+    for part in range(P):
+        shard, S = sp.slice_remap(dA, splits, part)
+        assert S == oracle.partition_slot(splits)
+        rp, col, val = oracle.slice_remap(A, splits, part)
+        assert np.array_equal(shard.row_ptr.cpu().numpy().astype(np.int64), rp)
+        assert np.array_equal(shard.col.cpu().numpy(), col)
+        assert np.array_equal(shard.val.cpu().numpy(), val)
+
+
+# ------------------------------------------------------------------ errors, semantics
+
+def test_not_canonical_rejected(sp):
+    A = case("u2048", "f64")
+    bad_cols = [A.col.copy() for _ in range(3)]
+    bad_cols[0][[3, 4]] = bad_cols[0][[4, 3]]              # unsorted within a row
+    bad_cols[1][5] = bad_cols[1][4]                         # duplicate
+    bad_cols[2][9] = A.n_cols                               # out of range
+    for c in bad_cols:
+        B = matgen.HostCSR(A.row_ptr, c, A.val, A.n_rows, A.n_cols)
+        dB = to_dev(sp, B, torch.float64)
+        with pytest.raises(sp.SpmvError) as e:
+            sp.features(dB)
+        assert e.value.status == 2
+        for fmt in ALL_FORMATS:
+            with pytest.raises(sp.SpmvError) as e:
+                sp.convert(dB, fmt)
+            assert e.value.status == 2
+    rp = A.row_ptr.copy()
+    rp[10], rp[11] = rp[11], rp[10]                         # non-monotone row_ptr
+    dB = to_dev(sp, matgen.HostCSR(rp, A.col, A.val, A.n_rows, A.n_cols), torch.float64)
+    with pytest.raises(sp.SpmvError) as e:
+        sp.convert(dB, "csr")
+    assert e.value.status == 2
+
+
+def test_ell_size_guard(sp):
+    A = case("rmat15", "f64")
+    with pytest.raises(sp.SpmvError) as e:
+        sp.convert(to_dev(sp, A, torch.float64), "ell")
+    assert e.value.status == 3
+    with pytest.raises(sp.SpmvError) as e:
+        sp.convert(to_dev(sp, case("u2048", "f64"), torch.float64), "ell", max_bytes=1000)
+    assert e.value.status == 3
+
+
+def test_x_y_overlap_rejected(sp):
+    A = matgen.uniform_fixed(64, 64, 4)
+    h = sp.convert(to_dev(sp, A, torch.float64), "csr")
+    buf = torch.zeros(64, dtype=torch.float64, device="cuda")
+    with pytest.raises(sp.SpmvError) as e:
+        h.run(1.0, buf, 0.0, buf)
+    assert e.value.status == 1
+
+
+@pytest.mark.parametrize("fmt", ALL_FORMATS)
+def test_deterministic_bits(sp, fmt):
+    A = case("rmat15", "f64")
+    dA = to_dev(sp, A, torch.float64)
+    if fmt == "ell":
+        pytest.skip("ELL infeasible on R-MAT")
+    x = matgen.vector(A.n_cols, 1, 1)
+    outs = []
+    for _ in range(3):
+        h, out = run_format(sp, A, dA, fmt, torch.float64, 1.0, 0.0, x, None)
+        outs.append(out)
+    assert all(np.array_equal(outs[0], o) for o in outs[1:])
+
+
+@pytest.mark.parametrize("fmt", ("csr", "merge", "csr5", "coo", "hyb"))
+def test_run_host_end_to_end(sp, fmt):
+    A = case("rmat12", "f64")
+    h = sp.convert(to_dev(sp, A, torch.float64), fmt)
+    x = matgen.vector(A.n_cols, 4, 1)
+    y = matgen.vector(A.n_rows, 4, 2)
+    ref, bound = oracle.spmv_csr(A, x, 2.0, 0.5, y, with_bound=True)
+    out = y.copy()
+    h.run_host(2.0, x, 0.5, out)
+    assert oracle.check_tolerance(out, ref, bound, 1e-12)[0]
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32], ids=["f64", "f32"])
+@pytest.mark.parametrize("fmt", ("csr", "merge", "csr5", "coo", "hyb", "ell"))
+def test_long_sequential_stress(sp, fmt, dtype):
+    """P9: positive non-dyadic values (0.1), x = 1, rows up to 1e6: the bound must hold
+    (catches long sequential fp32/fp64 accumulation chains, A13).  CSR-scalar is exempt:
+    one thread per row is the variant the paper describes, not a label."""
+    lens = np.array([1_000_000, 3, 30_000, 1, 250_000], np.int64)
+    n_cols = 1_000_000
+    rp = np.zeros(lens.size + 1, np.int64)
+    np.cumsum(lens, out=rp[1:])
+    col = np.concatenate([np.arange(l, dtype=np.int32) for l in lens])
+    A = matgen.HostCSR(rp, col, np.full(col.size, 0.1), lens.size, n_cols)
+    if dtype == torch.float32:
+        A = matgen.HostCSR(rp, col, np.full(col.size, float(np.float32(0.1))), lens.size, n_cols)
+    x = np.ones(n_cols)
+    ref, bound = oracle.spmv_csr(A, x, 1.0, 0.0, None, with_bound=True)
+    opts = {"max_bytes": 1 << 31} if fmt == "ell" else {}
+    h, out = run_format(sp, A, to_dev(sp, A, dtype), fmt, dtype, 1.0, 0.0, x, None, **opts)
+    ok, ratio, _ = oracle.check_tolerance(out, ref, bound, TOL[dtype])
+    assert ok, ratio
+
+
+# ------------------------------------------------------------------ full-size configs
+
+@pytest.mark.parametrize("fmt", ("coo", "ell", "csr", "hyb", "merge", "csr5"))
+def test_full_size_lap4096(sp, fmt):
+    """BASELINE configs[1] at full size, in the launch configuration bench.py times:
+    every row against the oracle (fp64, alpha=1, beta=1 with uniform x, y)."""
+    A = _lap4096()
+    x = matgen.vector(A.n_cols, matgen.SEEDS["lap4096"], 1)
+    y0 = matgen.vector(A.n_rows, matgen.SEEDS["lap4096"], 2)
+    ref, bound = _lap_ref(A, x, y0)
+    dA = _lap4096_dev(sp)
+    h, out = run_format(sp, A, dA, fmt, torch.float64, 1.0, 1.0, x, y0)
+    ok, ratio, nbad = oracle.check_tolerance(out, ref, bound, 1e-12)
+    assert ok, (fmt, nbad, ratio)
+
+
+_BIG = {}
+
+
+def _lap4096():
+    if "lap" not in _BIG:
+        _BIG["lap"] = matgen.laplacian5(4096)
+    return _BIG["lap"]
+
+
+def _lap4096_dev(sp):
+    if "lapd" not in _BIG:
+        _BIG["lapd"] = sp.CSR.from_host(_lap4096(), dtype=torch.float64)
+    return _BIG["lapd"]
+
+
+def _lap_ref(A, x, y0):
+    if "lapref" not in _BIG:
+        _BIG["lapref"] = oracle.spmv_csr(A, x, 1.0, 1.0, y0, with_bound=True)
+    return _BIG["lapref"]
