@@ -16,6 +16,7 @@ NVCC_FLAGS = [
     "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
     "--expt-relaxed-constexpr",
     "-Xptxas", "-warn-spills",
+    "-Xptxas", "-v",
 ]
 
 
@@ -45,17 +46,22 @@ def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -
     for src in sources():
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
         objs.append(obj)
-        cmd = ["nvcc", *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-dc", src, "-o", obj]
+        cmd = ["nvcc", *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]
         if verbose:
             print(" ".join(cmd))
         procs.append((src, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
     failed = []
+    logs = []
     for src, p in procs:
         out, _ = p.communicate()
         if p.returncode != 0:
             failed.append((src, out.decode()))
-        elif verbose and out:
-            print(out.decode())
+        else:
+            logs.append(out.decode())
+    with open(os.path.join(objdir, "ptxas.log"), "w") as f:
+        f.write("\n".join(logs))
+    if verbose:
+        print("ptxas report:", os.path.join(objdir, "ptxas.log"))
     if failed:
         raise RuntimeError("nvcc failed:\n" + "\n".join(f"{s}:\n{o}" for s, o in failed))
     tmp = LIB + f".tmp{os.getpid()}"

@@ -129,8 +129,11 @@ k_rows(const IT *__restrict__ rp, int64_t n_rows, int64_t nnz, int64_t kh,
     }
 }
 
-// F2: element pass, one warp per 32-position word -- column validity/order and the
-// block-start bitmap.
+// F2: element pass -- column validity/order and the block-start bitmap.  A warp
+// handles kWordsPerIter consecutive 32-position words per iteration (all loads
+// issued before any use: the pass is a pure stream over col_idx).
+constexpr int kWordsPerIter = 8;
+
 __global__ void __launch_bounds__(kThreads)
 k_flags(const int *__restrict__ col, int64_t nnz, int64_t n_cols, int64_t n_words,
         const unsigned *__restrict__ rs_bits, unsigned *__restrict__ flag_bits, FeatureSums *out) {
@@ -138,24 +141,36 @@ k_flags(const int *__restrict__ col, int64_t nnz, int64_t n_cols, int64_t n_word
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t n_warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const uint64_t pol = policy_evict_first();
-    unsigned long long bad = 0;
-    for (int64_t w = warp; w < n_words; w += n_warps) {
-        int64_t k = w * 32 + lane;
-        bool valid = k < nnz;
-        int c = valid ? ld_hint(col + k, pol) : 0;
-        int prev = __shfl_up_sync(0xffffffffu, c, 1);
-        if (lane == 0) prev = (k > 0 && valid) ? col[k - 1] : 0;
-        unsigned rs = rs_bits[w];
-        bool rowstart = (rs >> lane) & 1u;
-        bool flag = valid && (rowstart || k == 0 || (int64_t)c != (int64_t)prev + 1);
-        if (valid && (c < 0 || (int64_t)c >= n_cols)) bad |= BAD_COL_RANGE;
-        if (valid && k > 0 && !rowstart && c <= prev) bad |= BAD_COL_ORDER;
-        if (valid && k == 0 && !rowstart) bad |= BAD_ROWPTR_ORDER;
-        unsigned fw = __ballot_sync(0xffffffffu, flag);
-        if (lane == 0) flag_bits[w] = fw;
+    unsigned bad = 0;
+    for (int64_t wb = warp * kWordsPerIter; wb < n_words; wb += n_warps * kWordsPerIter) {
+        int c[kWordsPerIter];
+        unsigned rs[kWordsPerIter];
+#pragma unroll
+        for (int u = 0; u < kWordsPerIter; ++u) {
+            const int64_t k = (wb + u) * 32 + lane;
+            c[u] = k < nnz ? ld_hint(col + k, pol) : 0;
+            rs[u] = wb + u < n_words ? rs_bits[wb + u] : 0u;
+        }
+        const int64_t k0 = wb * 32;
+        int first_prev = (lane == 0 && k0 > 0 && k0 < nnz) ? col[k0 - 1] : 0;
+#pragma unroll
+        for (int u = 0; u < kWordsPerIter; ++u) {
+            const int64_t k = (wb + u) * 32 + lane;
+            const bool valid = k < nnz;
+            int prev = __shfl_up_sync(0xffffffffu, c[u], 1);
+            int last_prev_word = __shfl_sync(0xffffffffu, u > 0 ? c[u > 0 ? u - 1 : 0] : 0, 31);
+            if (lane == 0) prev = u == 0 ? first_prev : last_prev_word;
+            const bool rowstart = (rs[u] >> lane) & 1u;
+            const bool flag = valid && (rowstart || k == 0 || (int64_t)c[u] != (int64_t)prev + 1);
+            if (valid && (c[u] < 0 || (int64_t)c[u] >= n_cols)) bad |= BAD_COL_RANGE;
+            if (valid && k > 0 && !rowstart && c[u] <= prev) bad |= BAD_COL_ORDER;
+            if (valid && k == 0 && !rowstart) bad |= BAD_ROWPTR_ORDER;
+            const unsigned fw = __ballot_sync(0xffffffffu, flag);
+            if (lane == 0 && wb + u < n_words) flag_bits[wb + u] = fw;
+        }
     }
-    bad = __reduce_or_sync(0xffffffffu, (unsigned)bad);
-    if (lane == 0 && bad) atomicOr(&out->bad, bad);
+    bad = __reduce_or_sync(0xffffffffu, bad);
+    if (lane == 0 && bad) atomicOr(&out->bad, (unsigned long long)bad);
 }
 
 // F3a: per-chunk exclusive prefix of flag popcounts (kScanChunk words per block).
@@ -223,43 +238,54 @@ k_scan_totals(unsigned long long *totals, int64_t n) {
     }
 }
 
-// F4: block sizes = gaps between consecutive block starts (one warp per word).
+// F4: block sizes = gaps between consecutive block starts; kWordsPerIter words per
+// warp iteration (loaded up front), next start usually inside the batch, otherwise
+// a warp-cooperative forward scan (long contiguous blocks).
 __global__ void __launch_bounds__(kThreads)
 k_block_sizes(const unsigned *__restrict__ flag_bits, int64_t n_words, int64_t nnz, FeatureSums *out) {
     const int lane = threadIdx.x & 31;
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t n_warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     unsigned long long nb = 0, sz2 = 0, mn = ULLONG_MAX, mx = 0;
-    for (int64_t w = warp; w < n_words; w += n_warps) {
-        unsigned fw = flag_bits[w];
-        if (fw == 0) continue;                         // warp-uniform
-        // next block start after the word's last flag: usually in the next word,
-        // otherwise a warp-cooperative forward scan (long contiguous blocks)
-        int64_t next_after = nnz;
-        unsigned v1 = w + 1 < n_words ? flag_bits[w + 1] : 0u;
-        if (v1) {
-            next_after = (w + 1) * 32 + (__ffs(v1) - 1);
+    for (int64_t wb = warp * kWordsPerIter; wb < n_words; wb += n_warps * kWordsPerIter) {
+        unsigned fw[kWordsPerIter + 1];
+#pragma unroll
+        for (int u = 0; u <= kWordsPerIter; ++u) fw[u] = wb + u < n_words ? flag_bits[wb + u] : 0u;
+        // next block start at or after the batch end (only needed if the tail words are flag-free)
+        unsigned any = 0;
+#pragma unroll
+        for (int u = 0; u < kWordsPerIter; ++u) any |= fw[u];
+        if (!any) continue;                       // warp-uniform: no block starts in the batch
+        int64_t next_batch = nnz;
+        if (fw[kWordsPerIter]) {
+            next_batch = (wb + kWordsPerIter) * 32 + (__ffs(fw[kWordsPerIter]) - 1);
         } else {
-            for (int64_t base = w + 2; base < n_words; base += 32) {
+            for (int64_t base = wb + kWordsPerIter + 1; base < n_words; base += 32) {
                 unsigned v = base + lane < n_words ? flag_bits[base + lane] : 0u;
                 unsigned b = __ballot_sync(0xffffffffu, v != 0u);
                 if (b) {
                     int src = __ffs(b) - 1;
                     unsigned fv = __shfl_sync(0xffffffffu, v, src);
-                    next_after = (base + src) * 32 + (__ffs(fv) - 1);
+                    next_batch = (base + src) * 32 + (__ffs(fv) - 1);
                     break;
                 }
             }
         }
-        if ((fw >> lane) & 1u) {
-            unsigned above = lane == 31 ? 0u : (fw & ~((2u << lane) - 1u));
-            int64_t k = w * 32 + lane;
-            int64_t nxt = above ? w * 32 + (__ffs(above) - 1) : next_after;
-            unsigned long long s = (unsigned long long)(nxt - k);
-            nb += 1;
-            sz2 += s * s;
-            mn = s < mn ? s : mn;
-            mx = s > mx ? s : mx;
+        int64_t next_after = next_batch;          // next start after word u, scanning backwards
+#pragma unroll
+        for (int u = kWordsPerIter - 1; u >= 0; --u) {
+            const unsigned f = fw[u];
+            if ((f >> lane) & 1u) {
+                const unsigned above = lane == 31 ? 0u : (f & ~((2u << lane) - 1u));
+                const int64_t k = (wb + u) * 32 + lane;
+                const int64_t nxt = above ? (wb + u) * 32 + (__ffs(above) - 1) : next_after;
+                const unsigned long long sz = (unsigned long long)(nxt - k);
+                nb += 1;
+                sz2 += sz * sz;
+                mn = sz < mn ? sz : mn;
+                mx = sz > mx ? sz : mx;
+            }
+            if (f) next_after = (wb + u) * 32 + (__ffs(f) - 1);
         }
     }
     unsigned long long sums[2] = {nb, sz2};

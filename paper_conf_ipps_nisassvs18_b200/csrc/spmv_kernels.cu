@@ -75,47 +75,103 @@ __global__ void k_scale(V *y, int64_t n, double beta) {
 }
 
 // ------------------------------------------------------------------ CSR-vector (K3/G8)
-// "assign a WARP to process a row".  A W-lane group per row (A5);
-// lanes stride the row with four independent accumulators (folded every kFold
-// steps into a running total), shuffle reduction.
+// "assign a WARP to process a row".  A W-lane group per row (A5).
+// One warp iteration covers R = (32/W)*U consecutive rows: their row pointers come
+// from one coalesced load (+ shuffles), every group issues the first 2W elements of
+// each of its U rows before any x gather, and y is prefetched with the row
+// pointers, so a warp keeps ~2U independent loads per lane in flight even when
+// rows are as short as the 5-point stencil's.  Rows longer than 2W continue in a
+// four-accumulator loop folded every kFold steps (A13).
+template <int W> struct VecCfg { static constexpr int U = W <= 8 ? 4 : (W == 16 ? 2 : 1); };
+
 template <typename V, typename IT, int W, bool B0>
 __global__ void __launch_bounds__(kT)
 k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
              const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta) {
-    constexpr int RPW = 32 / W;
+    constexpr int G = 32 / W;
+    constexpr int U = (VecCfg<W>::U * G > 32) ? 32 / G : VecCfg<W>::U;
+    constexpr int R = G * U;                      // rows per warp iteration (<= 32)
     const int lane = threadIdx.x & 31;
     const int sub = lane & (W - 1);
+    const int g = lane / W;
     const int64_t gwarp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
-    for (int64_t base = gwarp * RPW; base < n; base += nwarps * RPW) {
-        const int64_t r = base + lane / W;
-        double tot = 0.0, a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;
-        if (r < n) {
-            const int64_t b = (int64_t)__ldg(rp + r + 1);
-            int64_t k = (int64_t)__ldg(rp + r) + sub;
+    for (int64_t base = gwarp * R; base < n; base += nwarps * R) {
+        const int64_t rp_lo = (int64_t)__ldg(rp + (base + lane < n ? base + lane : n));
+        const int64_t rp_hi = (int64_t)__ldg(rp + (base + R < n ? base + R : n));
+        double yv[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t r = base + u * G + g;
+            yv[u] = (!B0 && sub == 0 && r < n) ? (double)y[r] : 0.0;
+        }
+        int64_t a[U], b[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int i = u * G + g;                         // row index within the batch
+            a[u] = __shfl_sync(0xffffffffu, rp_lo, i);
+            const int64_t nx = __shfl_sync(0xffffffffu, rp_lo, (i + 1) & 31);
+            b[u] = i + 1 < R ? nx : rp_hi;
+            if (base + i >= n) { a[u] = 0; b[u] = 0; }
+        }
+        // first 2W elements of every row, all loads issued together
+        int c0[U], c1[U];
+        V v0[U], v1[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t k = a[u] + sub;
+            c0[u] = k < b[u] ? ld_hint(col + k, pa) : -1;
+            v0[u] = k < b[u] ? ld_hint(val + k, pa) : (V)0;
+            c1[u] = k + W < b[u] ? ld_hint(col + k + W, pa) : -1;
+            v1[u] = k + W < b[u] ? ld_hint(val + k + W, pa) : (V)0;
+        }
+        double s[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            double t0 = c0[u] >= 0 ? (double)v0[u] * (double)ld_x(x + c0[u], px) : 0.0;
+            double t1 = c1[u] >= 0 ? (double)v1[u] * (double)ld_x(x + c1[u], px) : 0.0;
+            s[u] = t0 + t1;
+        }
+        // long rows: the rest with four accumulators
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            int64_t k = a[u] + sub + 2 * W;
+            if (k >= b[u]) continue;
+            double tot = 0.0, a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;
             int it = 0;
-            for (; k + 3 * W < b; k += 4 * W) {
-                int c0 = ld_hint(col + k, pa), c1 = ld_hint(col + k + W, pa);
-                int c2 = ld_hint(col + k + 2 * W, pa), c3 = ld_hint(col + k + 3 * W, pa);
-                V v0 = ld_hint(val + k, pa), v1 = ld_hint(val + k + W, pa);
-                V v2 = ld_hint(val + k + 2 * W, pa), v3 = ld_hint(val + k + 3 * W, pa);
-                a0 += (double)v0 * (double)ld_x(x + c0, px);
-                a1 += (double)v1 * (double)ld_x(x + c1, px);
-                a2 += (double)v2 * (double)ld_x(x + c2, px);
-                a3 += (double)v3 * (double)ld_x(x + c3, px);
-                if (++it == kFold) {            // blocked summation keeps chains short (A13)
+            for (; k + 3 * W < b[u]; k += 4 * W) {
+                int d0 = ld_hint(col + k, pa), d1 = ld_hint(col + k + W, pa);
+                int d2 = ld_hint(col + k + 2 * W, pa), d3 = ld_hint(col + k + 3 * W, pa);
+                V w0 = ld_hint(val + k, pa), w1 = ld_hint(val + k + W, pa);
+                V w2 = ld_hint(val + k + 2 * W, pa), w3 = ld_hint(val + k + 3 * W, pa);
+                a0 += (double)w0 * (double)ld_x(x + d0, px);
+                a1 += (double)w1 * (double)ld_x(x + d1, px);
+                a2 += (double)w2 * (double)ld_x(x + d2, px);
+                a3 += (double)w3 * (double)ld_x(x + d3, px);
+                if (++it == kFold) {                     // blocked summation (A13)
                     tot += (a0 + a1) + (a2 + a3);
                     a0 = a1 = a2 = a3 = 0.0;
                     it = 0;
                 }
             }
-            for (; k < b; k += W) a0 += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
+            for (; k < b[u]; k += W) a0 += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
+            s[u] += tot + ((a0 + a1) + (a2 + a3));
         }
-        double s = tot + ((a0 + a1) + (a2 + a3));
 #pragma unroll
-        for (int o = W / 2; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-        if (sub == 0 && r < n) y_write<V, B0>(y, r, s, alpha, beta);
+        for (int u = 0; u < U; ++u) {
+#pragma unroll
+            for (int o = W / 2; o > 0; o >>= 1) s[u] += __shfl_xor_sync(0xffffffffu, s[u], o);
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t r = base + u * G + g;
+            if (sub == 0 && r < n) {
+                double o = alpha * s[u];
+                if (!B0) o = fma(beta, yv[u], o);
+                y[r] = (V)o;
+            }
+        }
     }
 }
 
@@ -127,6 +183,7 @@ k_csr_scalar(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
              const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta) {
     const uint64_t px = policy_evict_last();
     for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
+        const double yv = B0 ? 0.0 : (double)y[r];
         double a0 = 0.0, a1 = 0.0;
         int64_t k = __ldg(rp + r), b = __ldg(rp + r + 1);
         for (; k + 1 < b; k += 2) {
@@ -134,106 +191,164 @@ k_csr_scalar(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
             a1 += (double)__ldg(val + k + 1) * (double)ld_x(x + __ldg(col + k + 1), px);
         }
         if (k < b) a0 += (double)__ldg(val + k) * (double)ld_x(x + __ldg(col + k), px);
-        y_write<V, B0>(y, r, a0 + a1, alpha, beta);
+        double o = alpha * (a0 + a1);
+        if (!B0) o = fma(beta, yv, o);
+        y[r] = (V)o;
     }
 }
 
 // ------------------------------------------------------------------ ELL (K4/G9)
 // column-major, "each row is processed by a single thread".
-// Padding slots carry col = -1 and are skipped (A3).
+// Slots are consumed kEllBatch at a time with predicated loads (all in flight before
+// the first x gather); y is loaded before the slots.  Padding carries col = -1 (A3).
+constexpr int kEllBatch = 8;
+
 template <typename V, bool B0>
 __global__ void __launch_bounds__(kT)
 k_ell(const int *__restrict__ ecol, const V *__restrict__ eval, int64_t K, int64_t ld,
       const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta) {
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
     for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
-        double tot = 0.0, a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;
-        int64_t j = 0;
-        int it = 0;
-        for (; j + 3 < K; j += 4) {
-            int c0 = ld_hint(ecol + j * ld + r, pa), c1 = ld_hint(ecol + (j + 1) * ld + r, pa);
-            int c2 = ld_hint(ecol + (j + 2) * ld + r, pa), c3 = ld_hint(ecol + (j + 3) * ld + r, pa);
-            V v0 = ld_hint(eval + j * ld + r, pa), v1 = ld_hint(eval + (j + 1) * ld + r, pa);
-            V v2 = ld_hint(eval + (j + 2) * ld + r, pa), v3 = ld_hint(eval + (j + 3) * ld + r, pa);
-            if (c0 >= 0) a0 += (double)v0 * (double)ld_x(x + c0, px);
-            if (c1 >= 0) a1 += (double)v1 * (double)ld_x(x + c1, px);
-            if (c2 >= 0) a2 += (double)v2 * (double)ld_x(x + c2, px);
-            if (c3 >= 0) a3 += (double)v3 * (double)ld_x(x + c3, px);
-            if (++it == kFold) {
-                tot += (a0 + a1) + (a2 + a3);
-                a0 = a1 = a2 = a3 = 0.0;
-                it = 0;
+        const double yv = B0 ? 0.0 : (double)y[r];
+        double tot = 0.0, part = 0.0;
+        int nb = 0;
+        for (int64_t j0 = 0; j0 < K; j0 += kEllBatch) {
+            int c[kEllBatch];
+            V v[kEllBatch];
+#pragma unroll
+            for (int u = 0; u < kEllBatch; ++u) {
+                const bool in = j0 + u < K;
+                c[u] = in ? ld_hint(ecol + (j0 + u) * ld + r, pa) : -1;
+                v[u] = in ? ld_hint(eval + (j0 + u) * ld + r, pa) : (V)0;
+            }
+            double a0 = 0.0, a1 = 0.0;
+#pragma unroll
+            for (int u = 0; u < kEllBatch; u += 2) {
+                if (c[u] >= 0) a0 += (double)v[u] * (double)ld_x(x + c[u], px);
+                if (c[u + 1] >= 0) a1 += (double)v[u + 1] * (double)ld_x(x + c[u + 1], px);
+            }
+            part += a0 + a1;
+            if (++nb == kFold) {                          // blocked summation (A13)
+                tot += part;
+                part = 0.0;
+                nb = 0;
             }
         }
-        for (; j < K; ++j) {
-            int c = ld_hint(ecol + j * ld + r, pa);
-            V v = ld_hint(eval + j * ld + r, pa);
-            if (c >= 0) a0 += (double)v * (double)ld_x(x + c, px);
-        }
-        y_write<V, B0>(y, r, tot + ((a0 + a1) + (a2 + a3)), alpha, beta);
+        tot += part;
+        double o = alpha * tot;
+        if (!B0) o = fma(beta, yv, o);
+        y[r] = (V)o;
     }
 }
 
 // ------------------------------------------------------------------ COO (K1/G7)
 // "first all product contributions are computed for the non-zero
 // elements, followed by a segmented reduction across threads".  CTA c owns nonzeros
-// [c*T, (c+1)*T): staged products, thread-sequential segments of kIPT items, a
-// block segmented scan for the thread carries, a CTA carry for the fix-up.
-// ACCUM (HYB's COO part): y += alpha*s, no beta, no empty-row writes.
+// [c*T, (c+1)*T): row ids and products staged in shared memory (coalesced loads, all
+// x gathers of the chunk in flight), kIPT-item thread segments, a block segmented
+// scan for the thread carries, a CTA carry for the fix-up.  The chunk writes the
+// contiguous row window [R0, R1) (rows ending here + the empty rows before the next
+// chunk's first row): y of the window is prefetched into registers during staging
+// and written back coalesced; a window wider than kCooItems rows (huge gaps) spills
+// to direct writes.  ACCUM (HYB's COO part): y += alpha*s for the rows present only.
 template <typename V, bool ACCUM, bool B0>
 __global__ void __launch_bounds__(kT)
 k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restrict__ val, int64_t nnz,
       const V *__restrict__ x, V *__restrict__ y, int64_t n_rows, double alpha, double beta,
       int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
+    constexpr int kWin = (int)kCooItems;
     __shared__ int s_row[kCooItems + 1];
-    __shared__ double s_prod[kCooItems];
+    __shared__ double s_prod[kCooItems];            // products, then per-row sums
+    __shared__ unsigned s_mark[kCooItems / 32];
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
     const int64_t k0 = (int64_t)blockIdx.x * kCooItems;
     const int cnt = (int)(nnz - k0 < kCooItems ? nnz - k0 : kCooItems);
+    // row window of this chunk (uniform loads)
+    const int64_t R0 = (!ACCUM && blockIdx.x == 0) ? 0 : (int64_t)__ldg(row + k0);
+    const int64_t R1 = k0 + cnt < nnz ? (int64_t)__ldg(row + k0 + cnt) : n_rows;
+    const int64_t L = R1 - R0;
+    double yv[kIPT];
 #pragma unroll
     for (int u = 0; u < kIPT; ++u) {
-        int i = threadIdx.x + u * kT;
+        const int i = threadIdx.x + u * kT;
+        yv[u] = ((ACCUM || !B0) && i < L) ? (double)y[R0 + i] : 0.0;
+    }
+#pragma unroll
+    for (int u = 0; u < kIPT; ++u) {
+        const int i = threadIdx.x + u * kT;
         if (i < cnt) {
-            int c = ld_hint(col + k0 + i, pa);
-            V v = ld_hint(val + k0 + i, pa);
+            const int c = ld_hint(col + k0 + i, pa);
+            const V v = ld_hint(val + k0 + i, pa);
             s_row[i] = ld_hint(row + k0 + i, pa);
             s_prod[i] = (double)v * (double)ld_x(x + c, px);
         }
     }
-    if (threadIdx.x == 0) s_row[cnt] = k0 + cnt < nnz ? row[k0 + cnt] : (int)n_rows;   // sentinel
+    if (threadIdx.x < kCooItems / 32) s_mark[threadIdx.x] = 0u;
+    if (threadIdx.x == 0) s_row[cnt] = (int)R1;
     __syncthreads();
-    if (!ACCUM && blockIdx.x == 0 && threadIdx.x == 0)      // leading empty rows [0, row[0])
-        for (int r = 0; r < s_row[0]; ++r) y_beta<V, B0>(y, r, beta);
 
     const int i0 = threadIdx.x * kIPT;
     const int i1 = min(i0 + kIPT, cnt);
-    bool has_end = false;
-    double acc = 0.0, first_sum = 0.0;
-    int first_row = -1;
-    for (int i = i0; i < i1; ++i) {
-        acc += s_prod[i];
-        const int r = s_row[i], rn = s_row[i + 1];
-        if (rn != r) {                                   // row r ends at element i
-            if (!has_end) { first_sum = acc; first_row = r; has_end = true; }
-            else if (ACCUM) y[r] = (V)((double)y[r] + alpha * acc);
-            else y_write<V, B0>(y, r, acc, alpha, beta);
-            if (!ACCUM)
-                for (int g = r + 1; g < rn; ++g) y_beta<V, B0>(y, g, beta);   // empty rows in the gap
-            acc = 0.0;
+    unsigned emask = 0;
+    double ev[kIPT];
+    double acc = 0.0;
+#pragma unroll
+    for (int it = 0; it < kIPT; ++it) {
+        const int i = i0 + it;
+        ev[it] = 0.0;
+        if (i < i1) {
+            acc += s_prod[i];
+            const int r = s_row[i], rn = s_row[i + 1];
+            if (rn != r) {                                 // row r ends at element i
+                ev[it] = acc;
+                emask |= 1u << it;
+                acc = 0.0;
+                if (!ACCUM)                                // empty rows beyond the staged window
+                    for (int64_t gq = max((int64_t)r + 1, R0 + kWin); gq < rn; ++gq) y_beta<V, B0>(y, gq, beta);
+            }
         }
     }
     double incl;
-    const double carry_in = block_seg_scan(has_end || i0 >= cnt, i0 < cnt ? acc : 0.0, &incl);
-    if (has_end) {
-        const double s = first_sum + carry_in;
-        if (ACCUM) y[first_row] = (V)((double)y[first_row] + alpha * s);
-        else y_write<V, B0>(y, first_row, s, alpha, beta);
+    const double carry_in = block_seg_scan(emask != 0 || i0 >= cnt, i0 < cnt ? acc : 0.0, &incl);
+    bool first = true;
+#pragma unroll
+    for (int it = 0; it < kIPT; ++it) {
+        if ((emask >> it) & 1u) {
+            const double v = ev[it] + (first ? carry_in : 0.0);
+            first = false;
+            const int64_t r = s_row[i0 + it];
+            const int64_t li = r - R0;
+            if (li < kWin) {
+                s_prod[li] = v;
+                atomicOr(&s_mark[li >> 5], 1u << (li & 31));
+            } else if (ACCUM) {
+                y[r] = (V)((double)y[r] + alpha * v);
+            } else {
+                y_write<V, B0>(y, r, v, alpha, beta);
+            }
+        }
     }
-    // CTA carry: the thread holding the last element
-    if (i0 < cnt && i1 == cnt) {
+    if (i0 < cnt && i1 == cnt) {                           // CTA carry: the row open at the chunk end
         const bool open = s_row[cnt] == s_row[cnt - 1];
         carry_row[blockIdx.x] = open ? s_row[cnt - 1] : -1;
         carry_val[blockIdx.x] = open ? incl : 0.0;
+    }
+    if (!ACCUM && blockIdx.x == 0)                         // leading empty rows beyond the window
+        for (int64_t gq = kWin + threadIdx.x; gq < s_row[0]; gq += kT) y_beta<V, B0>(y, gq, beta);
+    __syncthreads();
+#pragma unroll
+    for (int u = 0; u < kIPT; ++u) {
+        const int i = threadIdx.x + u * kT;
+        if (i < L && i < kWin) {
+            const bool marked = (s_mark[i >> 5] >> (i & 31)) & 1u;
+            if (ACCUM) {
+                if (marked) y[R0 + i] = (V)(yv[u] + alpha * s_prod[i]);
+            } else {
+                double o = marked ? alpha * s_prod[i] : 0.0;
+                if (!B0) o = marked ? fma(beta, yv[u], o) : beta * yv[u];
+                y[R0 + i] = (V)o;
+            }
+        }
     }
 }
 
@@ -242,8 +357,10 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
 // rows into equal sized sub-problems".  CTA t consumes merge-path diagonals
 // [t*T, (t+1)*T) of (row ends) x (nonzeros) (coordinates precomputed at conversion,
 // A7).  Row ends and products are staged in shared memory with coalesced loads
-// (all x gathers of the tile in flight at once); each thread then consumes kIPT
-// consecutive items of the path.
+// (all x gathers of the tile in flight at once); y of the tile's rows [r0, r1) is
+// prefetched into registers at the same time.  Each thread consumes kIPT consecutive
+// path items; after the block segmented scan the per-row sums go to shared memory
+// and the tile writes y[r0, r1) coalesced.
 template <typename V, typename IT, bool B0>
 __global__ void __launch_bounds__(kT)
 k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
@@ -251,18 +368,28 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
         const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
         int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
     __shared__ int s_end[kMergeItems];
-    __shared__ double s_prod[kMergeItems];
+    __shared__ double s_prod[kMergeItems];          // products, then per-row sums
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
     const int64_t t = blockIdx.x;
     const int64_t r0 = crow[t], k0 = cnz[t], r1 = crow[t + 1], k1 = cnz[t + 1];
     const int nrows = (int)(r1 - r0), nnzt = (int)(k1 - k0), items = nrows + nnzt;
-    for (int i = threadIdx.x; i < nrows; i += kT) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
+    double yv[kIPT];
 #pragma unroll
     for (int u = 0; u < kIPT; ++u) {
-        int j = threadIdx.x + u * kT;
+        const int i = threadIdx.x + u * kT;
+        yv[u] = (!B0 && i < nrows) ? (double)y[r0 + i] : 0.0;
+    }
+#pragma unroll
+    for (int u = 0; u < kIPT; ++u) {
+        const int i = threadIdx.x + u * kT;
+        if (i < nrows) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
+    }
+#pragma unroll
+    for (int u = 0; u < kIPT; ++u) {
+        const int j = threadIdx.x + u * kT;
         if (j < nnzt) {
-            int c = ld_hint(col + k0 + j, pa);
-            V v = ld_hint(val + k0 + j, pa);
+            const int c = ld_hint(col + k0 + j, pa);
+            const V v = ld_hint(val + k0 + j, pa);
             s_prod[j] = (double)v * (double)ld_x(x + c, px);
         }
     }
@@ -272,44 +399,74 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
     const int nit = max(0, min(kIPT, items - d));
     int lo = max(0, d - nnzt), hi = min(d, nrows);
     while (lo < hi) {
-        int mid = (lo + hi + 1) >> 1;
+        const int mid = (lo + hi + 1) >> 1;
         if (s_end[mid - 1] + mid <= d) lo = mid; else hi = mid - 1;
     }
     int i = lo, j = d - lo;
-    bool has_end = false;
-    double acc = 0.0, first_sum = 0.0;
-    int64_t first_row = -1;
-    for (int it = 0; it < nit; ++it) {
-        if (i < nrows && s_end[i] <= j) {                // row r0+i ends (A7 tie-break)
-            if (!has_end) { first_sum = acc; first_row = r0 + i; has_end = true; }
-            else y_write<V, B0>(y, r0 + i, acc, alpha, beta);
-            acc = 0.0;
-            ++i;
-        } else {
-            acc += s_prod[j];
-            ++j;
+    const int first_local = i;
+    unsigned emask = 0;
+    double ev[kIPT];
+    double acc = 0.0;
+#pragma unroll
+    for (int it = 0; it < kIPT; ++it) {
+        ev[it] = 0.0;
+        if (it < nit) {
+            if (i < nrows && s_end[i] <= j) {              // row r0+i ends (A7 tie-break)
+                ev[it] = acc;
+                emask |= 1u << it;
+                acc = 0.0;
+                ++i;
+            } else {
+                acc += s_prod[j];
+                ++j;
+            }
         }
     }
     double incl;
-    const double carry_in = block_seg_scan(has_end || nit == 0, nit ? acc : 0.0, &incl);
-    if (has_end) y_write<V, B0>(y, first_row, first_sum + carry_in, alpha, beta);
+    const double carry_in = block_seg_scan(emask != 0 || nit == 0, nit ? acc : 0.0, &incl);
+    // (the scan's barriers guarantee every walk is done: s_prod is free for row sums)
+    int li = first_local;
+    bool first = true;
+#pragma unroll
+    for (int it = 0; it < kIPT; ++it) {
+        if ((emask >> it) & 1u) {
+            s_prod[li] = ev[it] + (first ? carry_in : 0.0);
+            first = false;
+            ++li;
+        }
+    }
     // tile carry: nonzeros after the tile's last row end belong to row r1 (ends later)
     if (nit > 0 && d + nit == items) {
         const bool open = r1 < n_rows && k1 > (nrows ? k0 + s_end[nrows - 1] : k0);
         carry_row[t] = open ? r1 : -1;
         carry_val[t] = open ? incl : 0.0;
     }
-    if (items == 0 && threadIdx.x == 0) carry_row[t] = -1;
+    __syncthreads();
+#pragma unroll
+    for (int u = 0; u < kIPT; ++u) {
+        const int q = threadIdx.x + u * kT;
+        if (q < nrows) {
+            double o = alpha * s_prod[q];
+            if (!B0) o = fma(beta, yv[u], o);
+            y[r0 + q] = (V)o;
+        }
+    }
 }
 
 // ------------------------------------------------------------------ CSR5 (K6/G12)
 // equally sized 2-D tiles (32 lanes x sigma) with tile_ptr and
 // tile_desc.  One warp per tile.  Lane l holds elements t*W + l*sigma + s stored
 // lane-interleaved (A6) so each lane issues 16-byte loads.  Segments (rows) closed
-// inside a lane are written directly; the segment a lane opens last is completed by
-// a flag-segmented suffix sum of the next lanes' heads (shuffles; y_offset gives the
-// segment index, the empty-row map or row_lo gives its row).  The tile's leading
-// partial (row tile_ptr[t], started in an earlier tile) is the tile carry.
+// inside a lane are finished in-lane; the segment a lane opens last is completed by a
+// flag-segmented suffix sum of the next lanes' heads (shuffles; y_offset gives the
+// segment index, the empty-row map or row_lo gives its row).  The tile emits exactly
+// the rows [row_lo[t], row_lo[t+1]): y of that window (up to kCsr5Win rows) is
+// prefetched while the x gathers are in flight, the row sums are collected in a
+// per-warp shared buffer and the window is written back coalesced (empty rows get
+// beta*y).  The tile's leading partial (row tile_ptr[t], started in an earlier tile)
+// is the tile carry.
+constexpr int kCsr5Win = 128;
+
 template <int SIGMA, typename V>
 struct Csr5Vec;
 template <int SIGMA>
@@ -343,7 +500,10 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
        const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
        int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
     constexpr int64_t W = 32 * SIGMA;
-    const int lane = threadIdx.x & 31;
+    constexpr int kQ = kCsr5Win / 32;
+    __shared__ double s_acc[kT / 32][kCsr5Win];
+    __shared__ unsigned s_mark[kT / 32][kCsr5Win / 32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     if (t > n_tiles) return;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
@@ -367,6 +527,8 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
     }
     const int64_t base = t * W;
     const unsigned d = __ldg(desc + t * 32 + lane);
+    const int64_t lo = __ldg(row_lo + t), hi = __ldg(row_lo + t + 1);
+    const int64_t moff = __ldg(map_off + t);
     int c[SIGMA];
 #pragma unroll
     for (int q = 0; q < SIGMA / 4; ++q) {
@@ -375,15 +537,32 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
     }
     V v[SIGMA];
     Csr5Vec<SIGMA, V>::load(val, base, lane, v, pa);
+    const int64_t L = hi - lo;
+    double yv[kQ];
+#pragma unroll
+    for (int q = 0; q < kQ; ++q) {
+        const int i = lane + 32 * q;
+        yv[q] = (!B0 && i < L) ? (double)y[lo + i] : 0.0;
+    }
+    if (lane < kCsr5Win / 32) s_mark[wid][lane] = 0u;
     double p[SIGMA];
 #pragma unroll
     for (int s = 0; s < SIGMA; ++s) p[s] = (double)v[s] * (double)ld_x(x + c[s], px);
+    __syncwarp();
 
     const unsigned flag = d & 0xFFFFu;
     const int y_off = (int)((d >> 16) & 0x1FFu);
-    const int64_t lo = __ldg(row_lo + t);
-    const int64_t moff = __ldg(map_off + t);
     auto seg_row = [&](int idx) -> int64_t { return moff >= 0 ? __ldg(seg_map + moff + idx) : lo + idx; };
+    auto emit = [&](int idx, double sum) {
+        const int64_t r = seg_row(idx);
+        const int64_t li = r - lo;
+        if (li < kCsr5Win) {
+            s_acc[wid][li] = sum;
+            atomicOr(&s_mark[wid][li >> 5], 1u << (li & 31));
+        } else {
+            y_write<V, B0>(y, r, sum, alpha, beta);
+        }
+    };
 
     double acc = 0.0, head = 0.0;
     int kseg = 0;
@@ -391,7 +570,7 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
     for (int s = 0; s < SIGMA; ++s) {
         if ((flag >> s) & 1u) {
             if (kseg == 0) head = acc;
-            else y_write<V, B0>(y, seg_row(y_off + kseg - 1), acc, alpha, beta);   // closed in-lane
+            else emit(y_off + kseg - 1, acc);              // segment closed inside the lane
             ++kseg;
             acc = 0.0;
         }
@@ -403,8 +582,8 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
     bool F = kseg > 0;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-        double Rn = __shfl_down_sync(0xffffffffu, R, o);
-        int Fn = __shfl_down_sync(0xffffffffu, (int)F, o);
+        const double Rn = __shfl_down_sync(0xffffffffu, R, o);
+        const int Fn = __shfl_down_sync(0xffffffffu, (int)F, o);
         if (!F) {
             if (lane + o < 32) { R += Rn; F = Fn; }
             else F = true;
@@ -412,15 +591,26 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
     }
     double Rnext = __shfl_down_sync(0xffffffffu, R, 1);
     if (lane == 31) Rnext = 0.0;
-    if (kseg > 0) y_write<V, B0>(y, seg_row(y_off + kseg - 1), acc + Rnext, alpha, beta);
+    if (kseg > 0) emit(y_off + kseg - 1, acc + Rnext);
     if (lane == 0) {
         const bool lead = !(flag & 1u);
         carry_row[t] = lead ? __ldg(tile_ptr + t) : -1;
         carry_val[t] = lead ? R : 0.0;
     }
-    if (moff >= 0) {                                     // empty rows of the tile's range
-        const int64_t hi = __ldg(row_lo + t + 1);
-        for (int64_t r = lo + lane; r < hi; r += 32)
+    __syncwarp();
+    // write the window: segment rows alpha*s + beta*y, empty rows beta*y
+#pragma unroll
+    for (int q = 0; q < kQ; ++q) {
+        const int i = lane + 32 * q;
+        if (i < L) {
+            const bool marked = (s_mark[wid][i >> 5] >> (i & 31)) & 1u;
+            double o = marked ? alpha * s_acc[wid][i] : 0.0;
+            if (!B0) o = marked ? fma(beta, yv[q], o) : beta * yv[q];
+            y[lo + i] = (V)o;
+        }
+    }
+    if (L > kCsr5Win && moff >= 0) {                       // empty rows beyond the window
+        for (int64_t r = lo + kCsr5Win + lane; r < hi; r += 32)
             if (__ldg(rp + r + 1) == __ldg(rp + r)) y_beta<V, B0>(y, r, beta);
     }
 }
