@@ -136,8 +136,8 @@ typedef struct {
     int vector_width;      /* CSR-vector lanes per row (0 = A5 rule), power of two 1..32  */
     size_t max_bytes;      /* ELL/HYB guard (0 = min(1/2 free memory, max(8x the CSR bytes,
                               64 MiB)))                                                    */
-    int alias_input;       /* 1 = COO/CSR/MERGE handles reference the caller's col/vals
-                              (caller keeps them alive and unchanged)                     */
+    int alias_input;       /* 1 = COO/CSR handles reference the caller's col/vals (caller
+                              keeps them alive and unchanged); MERGE/CSR5/ELL/HYB copy     */
 } spmv_convert_opts;
 
 /* Fill `opts` with the defaults (all rules as above). */

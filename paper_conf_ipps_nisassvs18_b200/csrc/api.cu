@@ -284,7 +284,7 @@ spmv_status spmv_destroy(spmv_handle *h, void *stream) {
     if (!h) return SPMV_OK;
     cudaStream_t s = as_stream(stream);
     for (int i = 0; i < kMaxArrays; ++i)
-        if (h->arr[i].owned && h->arr[i].p) dev_free(h->ctx, h->arr[i].p, h->arr[i].bytes, s);
+        if (h->arr[i].owned && h->arr[i].p) dev_free(h->ctx, h->arr[i].p, h->arr[i].bytes + 64, s);
     dev_free(h->ctx, h->carry_row.p, h->carry_row.bytes, s);
     dev_free(h->ctx, h->carry_val.p, h->carry_val.bytes, s);
     dev_free(h->ctx, h->io_x.p, h->io_x.bytes, s);

@@ -191,12 +191,18 @@ int grid_cap(const spmv_ctx *ctx, int64_t work) {
     return (int)std::max<int64_t>(1, std::min(g, cap));
 }
 
+// Handle arrays carry kArrayPad bytes of slack so that vector loads of a lane chunk
+// shifted to 16-byte alignment (merge kernel) never leave the allocation.
+constexpr size_t kArrayPad = 64;
+
 spmv_status arr_alloc(spmv_handle *h, int id, size_t bytes, cudaStream_t s) {
     DevArray &a = h->arr[id];
     a.bytes = bytes;
     a.owned = true;
     if (bytes == 0) { a.p = nullptr; return SPMV_OK; }
-    return dev_alloc(h->ctx, bytes, s, &a.p);
+    SPMV_TRY(dev_alloc(h->ctx, bytes + kArrayPad, s, &a.p));
+    SPMV_CUDA_TRY(cudaMemsetAsync((char *)a.p + bytes, 0, kArrayPad, s));
+    return SPMV_OK;
 }
 
 template <typename IT, typename V>
@@ -357,7 +363,7 @@ spmv_status convert_t(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, const s
         break;
     }
     case SPMV_MERGE: {
-        SPMV_TRY(copy_colval(o->alias_input != 0));
+        SPMV_TRY(copy_colval(false));   // padded copies: the kernel's shifted vector loads need the slack
         int64_t T = o->merge_items > 0 ? o->merge_items : kMergeItems;
         if (T != kMergeItems) {
             set_error("merge_items other than the compiled tile size is not supported");

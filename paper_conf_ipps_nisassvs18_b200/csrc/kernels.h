@@ -5,6 +5,7 @@
 namespace spmv {
 constexpr int kRunThreads = 256;           // CTA size of the tiled kernels
 constexpr int kItemsPerThread = 8;         // sequential items per thread (COO / merge)
-constexpr int64_t kCooItems = kRunThreads * kItemsPerThread;     // nonzeros per COO CTA
-constexpr int64_t kMergeItems = kRunThreads * kItemsPerThread;   // merge-path items per CTA
+constexpr int kWarpItemsPerLane = 8;      // sequential items per lane (warp-tile COO / merge)
+constexpr int64_t kCooItems = 32 * kWarpItemsPerLane;     // nonzeros per COO warp tile
+constexpr int64_t kMergeItems = 32 * kWarpItemsPerLane;   // merge-path items per warp tile
 }  // namespace spmv

@@ -12,6 +12,7 @@
 // y = alpha*s + beta*y, earlier CTAs leave (row, partial) carries that k_fixup adds
 // in carry order (one thread per run of equal rows).
 #include <algorithm>
+#include <climits>
 
 #include "internal.h"
 #include "kernels.h"
@@ -22,38 +23,11 @@ namespace {
 
 constexpr int kT = kRunThreads;
 constexpr int kIPT = kItemsPerThread;
+constexpr int kWIPT = kWarpItemsPerLane;
+constexpr int kMinBlocks = 4;   // 4 CTAs x 256 threads per SM: <= 64 registers
 constexpr int kFold = 256;   // sequential steps per accumulator before folding (A13)
 
 // ------------------------------------------------------------------ helpers
-
-// Block-wide segmented scan over threads (kT threads): S(t) = v(t) + (head(t) ? 0 : S(t-1)).
-// Returns the exclusive value S(t-1) (0 for t = 0); *incl receives S(t).
-__device__ __forceinline__ double block_seg_scan(bool head, double v, double *incl) {
-    __shared__ double s_S[kT / 32];
-    __shared__ int s_H[kT / 32];
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    double S = v;
-    bool H = head;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        double Sp = __shfl_up_sync(0xffffffffu, S, o);
-        int Hp = __shfl_up_sync(0xffffffffu, (int)H, o);
-        if (lane >= o) {
-            if (!H) S += Sp;
-            H = H || Hp;
-        }
-    }
-    if (lane == 31) { s_S[wid] = S; s_H[wid] = H; }
-    __syncthreads();
-    double carry = 0.0;                     // combination of warps < wid
-    for (int w = 0; w < wid; ++w) carry = s_H[w] ? s_S[w] : carry + s_S[w];
-    double full = H ? S : S + carry;
-    double ex = __shfl_up_sync(0xffffffffu, full, 1);
-    if (lane == 0) ex = carry;
-    __syncthreads();
-    *incl = full;
-    return ex;
-}
 
 template <typename V, bool B0>
 __device__ __forceinline__ void y_write(V *y, int64_t r, double s, double alpha, double beta) {
@@ -76,16 +50,16 @@ __global__ void k_scale(V *y, int64_t n, double beta) {
 
 // ------------------------------------------------------------------ CSR-vector (K3/G8)
 // "assign a WARP to process a row".  A W-lane group per row (A5).
-// One warp iteration covers R = (32/W)*U consecutive rows: their row pointers come
-// from one coalesced load (+ shuffles), every group issues the first 2W elements of
-// each of its U rows before any x gather, and y is prefetched with the row
-// pointers, so a warp keeps ~2U independent loads per lane in flight even when
-// rows are as short as the 5-point stencil's.  Rows longer than 2W continue in a
-// four-accumulator loop folded every kFold steps (A13).
-template <int W> struct VecCfg { static constexpr int U = W <= 8 ? 4 : (W == 16 ? 2 : 1); };
+// One warp iteration covers R = 32 consecutive rows (U = W rows per group): their row
+// pointers come from one coalesced load (+ shuffles) issued one iteration ahead
+// (software pipelined), and every group issues the first W elements of each of its U
+// rows before any x gather, so a warp keeps U independent loads per lane in flight
+// even when rows are as short as the 5-point stencil's.  Rows longer than W continue
+// in a four-accumulator loop folded every kFold steps (A13).
+template <int W> struct VecCfg { static constexpr int U = W <= 8 ? 32 / (32 / W) : (W == 16 ? 4 : 2); };
 
 template <typename V, typename IT, int W, bool B0>
-__global__ void __launch_bounds__(kT)
+__global__ void __launch_bounds__(kT, 3)
 k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
              const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta) {
     constexpr int G = 32 / W;
@@ -97,78 +71,89 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
     const int64_t gwarp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
-    for (int64_t base = gwarp * R; base < n; base += nwarps * R) {
-        const int64_t rp_lo = (int64_t)__ldg(rp + (base + lane < n ? base + lane : n));
-        const int64_t rp_hi = (int64_t)__ldg(rp + (base + R < n ? base + R : n));
-        double yv[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-            const int64_t r = base + u * G + g;
-            yv[u] = (!B0 && sub == 0 && r < n) ? (double)y[r] : 0.0;
+    int64_t base = gwarp * R;
+    IT nlo = 0, nhi = 0;                          // row pointers of the next batch (prefetched)
+    if (base < n) {
+        nlo = __ldg(rp + (base + lane < n ? base + lane : n));
+        nhi = __ldg(rp + (base + R < n ? base + R : n));
+    }
+    for (; base < n; base += nwarps * R) {
+        const IT rp_lo = nlo, rp_hi = nhi;
+        const int64_t nb = base + nwarps * R;
+        if (nb < n) {                             // issue the next batch's row pointers now
+            nlo = __ldg(rp + (nb + lane < n ? nb + lane : n));
+            nhi = __ldg(rp + (nb + R < n ? nb + R : n));
         }
-        int64_t a[U], b[U];
+        IT a[U], b[U];
 #pragma unroll
         for (int u = 0; u < U; ++u) {
             const int i = u * G + g;                         // row index within the batch
             a[u] = __shfl_sync(0xffffffffu, rp_lo, i);
-            const int64_t nx = __shfl_sync(0xffffffffu, rp_lo, (i + 1) & 31);
+            const IT nx = __shfl_sync(0xffffffffu, rp_lo, (i + 1) & 31);
             b[u] = i + 1 < R ? nx : rp_hi;
             if (base + i >= n) { a[u] = 0; b[u] = 0; }
         }
-        // first 2W elements of every row, all loads issued together
-        int c0[U], c1[U];
-        V v0[U], v1[U];
+        // first W elements of every row, all loads issued together
+        int c0[U];
+        V v0[U];
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-            const int64_t k = a[u] + sub;
+            const int64_t k = (int64_t)a[u] + sub;
             c0[u] = k < b[u] ? ld_hint(col + k, pa) : -1;
             v0[u] = k < b[u] ? ld_hint(val + k, pa) : (V)0;
-            c1[u] = k + W < b[u] ? ld_hint(col + k + W, pa) : -1;
-            v1[u] = k + W < b[u] ? ld_hint(val + k + W, pa) : (V)0;
         }
         double s[U];
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-            double t0 = c0[u] >= 0 ? (double)v0[u] * (double)ld_x(x + c0[u], px) : 0.0;
-            double t1 = c1[u] >= 0 ? (double)v1[u] * (double)ld_x(x + c1[u], px) : 0.0;
-            s[u] = t0 + t1;
-        }
-        // long rows: the rest with four accumulators
+        for (int u = 0; u < U; ++u) s[u] = c0[u] >= 0 ? (double)v0[u] * (double)ld_x(x + c0[u], px) : 0.0;
+        // longer rows: the rest with four accumulators (warp-uniform skip when none)
+        bool more = false;
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-            int64_t k = a[u] + sub + 2 * W;
-            if (k >= b[u]) continue;
-            double tot = 0.0, a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;
-            int it = 0;
-            for (; k + 3 * W < b[u]; k += 4 * W) {
-                int d0 = ld_hint(col + k, pa), d1 = ld_hint(col + k + W, pa);
-                int d2 = ld_hint(col + k + 2 * W, pa), d3 = ld_hint(col + k + 3 * W, pa);
-                V w0 = ld_hint(val + k, pa), w1 = ld_hint(val + k + W, pa);
-                V w2 = ld_hint(val + k + 2 * W, pa), w3 = ld_hint(val + k + 3 * W, pa);
-                a0 += (double)w0 * (double)ld_x(x + d0, px);
-                a1 += (double)w1 * (double)ld_x(x + d1, px);
-                a2 += (double)w2 * (double)ld_x(x + d2, px);
-                a3 += (double)w3 * (double)ld_x(x + d3, px);
-                if (++it == kFold) {                     // blocked summation (A13)
-                    tot += (a0 + a1) + (a2 + a3);
-                    a0 = a1 = a2 = a3 = 0.0;
-                    it = 0;
+        for (int u = 0; u < U; ++u) more |= (int64_t)a[u] + W < (int64_t)b[u];
+        if (__any_sync(0xffffffffu, more)) {
+#pragma unroll 1
+            for (int u = 0; u < U; ++u) {
+                const int i = u * G + g;
+                const IT au = __shfl_sync(0xffffffffu, rp_lo, i);
+                const IT nx = __shfl_sync(0xffffffffu, rp_lo, (i + 1) & 31);
+                const int64_t bu = base + i < n ? (int64_t)(i + 1 < R ? nx : rp_hi) : 0;
+                int64_t k = (int64_t)au + sub + W;
+                double tot = 0.0, a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;
+                int it = 0;
+                for (; k + 3 * W < bu; k += 4 * W) {
+                    int d0 = ld_hint(col + k, pa), d1 = ld_hint(col + k + W, pa);
+                    int d2 = ld_hint(col + k + 2 * W, pa), d3 = ld_hint(col + k + 3 * W, pa);
+                    V w0 = ld_hint(val + k, pa), w1 = ld_hint(val + k + W, pa);
+                    V w2 = ld_hint(val + k + 2 * W, pa), w3 = ld_hint(val + k + 3 * W, pa);
+                    a0 += (double)w0 * (double)ld_x(x + d0, px);
+                    a1 += (double)w1 * (double)ld_x(x + d1, px);
+                    a2 += (double)w2 * (double)ld_x(x + d2, px);
+                    a3 += (double)w3 * (double)ld_x(x + d3, px);
+                    if (++it == kFold) {                 // blocked summation (A13)
+                        tot += (a0 + a1) + (a2 + a3);
+                        a0 = a1 = a2 = a3 = 0.0;
+                        it = 0;
+                    }
                 }
+                for (; k < bu; k += W) a0 += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
+                const double extra = tot + ((a0 + a1) + (a2 + a3));
+#pragma unroll
+                for (int uu = 0; uu < U; ++uu) s[uu] += (uu == u) ? extra : 0.0;
             }
-            for (; k < b[u]; k += W) a0 += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
-            s[u] += tot + ((a0 + a1) + (a2 + a3));
         }
 #pragma unroll
         for (int u = 0; u < U; ++u) {
 #pragma unroll
             for (int o = W / 2; o > 0; o >>= 1) s[u] += __shfl_xor_sync(0xffffffffu, s[u], o);
         }
+        // the group's U results: lane sub == u of group g writes row u*G + g
+        double mine = 0.0;
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-            const int64_t r = base + u * G + g;
-            if (sub == 0 && r < n) {
-                double o = alpha * s[u];
-                if (!B0) o = fma(beta, yv[u], o);
+        for (int u = 0; u < U; ++u) mine = (sub == u) ? s[u] : mine;
+        if (sub < U) {
+            const int64_t r = base + sub * G + g;
+            if (r < n) {
+                double o = alpha * mine;
+                if (!B0) o = fma(beta, (double)y[r], o);
                 y[r] = (V)o;
             }
         }
@@ -241,112 +226,193 @@ k_ell(const int *__restrict__ ecol, const V *__restrict__ eval, int64_t K, int64
     }
 }
 
+// ------------------------------------------------------------------ warp-tile helpers
+
+// cp.async (LDGSTS): global -> shared without staging in registers
+template <int B>
+__device__ __forceinline__ void cp_async_n(void *smem, const void *gmem) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(s), "l"(gmem), "n"(B));
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
+// Flag-segmented suffix sum over the 32 lanes (CSR5's cross-lane step):
+// R[l] = head[l] + (F[l] ? 0 : R[l+1]), F[l] = "lane l holds a segment start".
+// Returns R[l+1] (0 for lane 31) in *Rnext and R[l].
+__device__ __forceinline__ double seg_suffix(double head, bool flagged, double *Rnext) {
+    const int lane = threadIdx.x & 31;
+    double R = head;
+    int F = flagged;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const double Rn = __shfl_down_sync(0xffffffffu, R, o);
+        const int Fn = __shfl_down_sync(0xffffffffu, F, o);
+        if (!F) {
+            if (lane + o < 32) { R += Rn; F = Fn; }
+            else F = 1;
+        }
+    }
+    const double rn = __shfl_down_sync(0xffffffffu, R, 1);
+    *Rnext = lane == 31 ? 0.0 : rn;
+    return R;
+}
+
+// Per-warp output window: row sums land in shared memory, then the window
+// [lo, lo+L) is written back coalesced (y prefetched in registers, kOutQ per lane).
+constexpr int kOutWin = 128;
+constexpr int kOutQ = kOutWin / 32;
+
 // ------------------------------------------------------------------ COO (K1/G7)
 // "first all product contributions are computed for the non-zero
-// elements, followed by a segmented reduction across threads".  CTA c owns nonzeros
-// [c*T, (c+1)*T): row ids and products staged in shared memory (coalesced loads, all
-// x gathers of the chunk in flight), kIPT-item thread segments, a block segmented
-// scan for the thread carries, a CTA carry for the fix-up.  The chunk writes the
-// contiguous row window [R0, R1) (rows ending here + the empty rows before the next
-// chunk's first row): y of the window is prefetched into registers during staging
-// and written back coalesced; a window wider than kCooItems rows (huge gaps) spills
-// to direct writes.  ACCUM (HYB's COO part): y += alpha*s for the rows present only.
-template <typename V, bool ACCUM, bool B0>
-__global__ void __launch_bounds__(kT)
-k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restrict__ val, int64_t nnz,
-      const V *__restrict__ x, V *__restrict__ y, int64_t n_rows, double alpha, double beta,
-      int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
-    constexpr int kWin = (int)kCooItems;
-    __shared__ int s_row[kCooItems + 1];
-    __shared__ double s_prod[kCooItems];            // products, then per-row sums
-    __shared__ unsigned s_mark[kCooItems / 32];
-    const uint64_t pa = policy_evict_first(), px = policy_evict_last();
-    const int64_t k0 = (int64_t)blockIdx.x * kCooItems;
-    const int cnt = (int)(nnz - k0 < kCooItems ? nnz - k0 : kCooItems);
-    // row window of this chunk (uniform loads)
-    const int64_t R0 = (!ACCUM && blockIdx.x == 0) ? 0 : (int64_t)__ldg(row + k0);
-    const int64_t R1 = k0 + cnt < nnz ? (int64_t)__ldg(row + k0 + cnt) : n_rows;
-    const int64_t L = R1 - R0;
-    double yv[kIPT];
+// elements, followed by a segmented reduction across threads".  One warp owns a tile
+// of 32 x kWIPT consecutive nonzeros, lane l the kWIPT consecutive elements
+// [8l, 8l+8): row/col/val arrive with 16-byte vector loads straight into registers,
+// all x gathers in flight together.  A new segment starts wherever the row id
+// changes; segments closed inside a lane are finished in-lane, the last one a lane
+// opens is completed by the flag-segmented suffix sum over lanes (as in CSR5).
+// Rows that START in the tile are written by it (alpha*s + beta*y); a leading
+// continuation of a row started in an earlier tile is the tile carry (fix-up); empty
+// rows between the tile's rows and up to the next tile's first row get beta*y.  The
+// tile's row window is staged in shared memory and written back coalesced.
+// ACCUM (HYB's COO part): y += alpha*s for rows present, nothing else.
+template <typename V> struct VecLoad8;
+template <> struct VecLoad8<double> {
+    static __device__ __forceinline__ void load(const double *p, double (&v)[8], uint64_t pol) {
 #pragma unroll
-    for (int u = 0; u < kIPT; ++u) {
-        const int i = threadIdx.x + u * kT;
-        yv[u] = ((ACCUM || !B0) && i < L) ? (double)y[R0 + i] : 0.0;
-    }
-#pragma unroll
-    for (int u = 0; u < kIPT; ++u) {
-        const int i = threadIdx.x + u * kT;
-        if (i < cnt) {
-            const int c = ld_hint(col + k0 + i, pa);
-            const V v = ld_hint(val + k0 + i, pa);
-            s_row[i] = ld_hint(row + k0 + i, pa);
-            s_prod[i] = (double)v * (double)ld_x(x + c, px);
+        for (int q = 0; q < 4; ++q) {
+            double2 w = ld_hint(reinterpret_cast<const double2 *>(p) + q, pol);
+            v[2 * q] = w.x; v[2 * q + 1] = w.y;
         }
     }
-    if (threadIdx.x < kCooItems / 32) s_mark[threadIdx.x] = 0u;
-    if (threadIdx.x == 0) s_row[cnt] = (int)R1;
-    __syncthreads();
+};
+template <> struct VecLoad8<float> {
+    static __device__ __forceinline__ void load(const float *p, float (&v)[8], uint64_t pol) {
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+            float4 w = ld_hint(reinterpret_cast<const float4 *>(p) + q, pol);
+            v[4 * q] = w.x; v[4 * q + 1] = w.y; v[4 * q + 2] = w.z; v[4 * q + 3] = w.w;
+        }
+    }
+};
+__device__ __forceinline__ void load_int8(const int *p, int (&v)[8], uint64_t pol) {
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+        int4 w = ld_hint(reinterpret_cast<const int4 *>(p) + q, pol);
+        v[4 * q] = w.x; v[4 * q + 1] = w.y; v[4 * q + 2] = w.z; v[4 * q + 3] = w.w;
+    }
+}
 
-    const int i0 = threadIdx.x * kIPT;
-    const int i1 = min(i0 + kIPT, cnt);
-    unsigned emask = 0;
-    double ev[kIPT];
-    double acc = 0.0;
+template <typename V, bool ACCUM, bool B0>
+__global__ void __launch_bounds__(kT, kMinBlocks)
+k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restrict__ val, int64_t nnz,
+      int64_t n_tiles, const V *__restrict__ x, V *__restrict__ y, int64_t n_rows, double alpha, double beta,
+      int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
+    static_assert(kWIPT == 8, "COO lane chunk is 8 elements");
+    __shared__ double s_acc_all[kT / 32][kOutWin];
+    __shared__ unsigned s_mark_all[kT / 32][kOutWin / 32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    if (t >= n_tiles) return;
+    double *s_acc = s_acc_all[wid];
+    unsigned *s_mark = s_mark_all[wid];
+    const uint64_t pa = policy_evict_first(), px = policy_evict_last();
+    const int64_t k0 = t * kCooItems;
+    const int cnt = (int)(nnz - k0 < kCooItems ? nnz - k0 : kCooItems);
+    const int64_t e0 = k0 + lane * 8;
+    const int nv = max(0, min(8, cnt - lane * 8));           // valid elements of this lane
+    int r[8], c[8];
+    V v[8];
+    if (cnt == (int)kCooItems) {
+        load_int8(row + e0, r, pa);
+        load_int8(col + e0, c, pa);
+        VecLoad8<V>::load(val + e0, v, pa);
+    } else {
 #pragma unroll
-    for (int it = 0; it < kIPT; ++it) {
-        const int i = i0 + it;
-        ev[it] = 0.0;
-        if (i < i1) {
-            acc += s_prod[i];
-            const int r = s_row[i], rn = s_row[i + 1];
-            if (rn != r) {                                 // row r ends at element i
-                ev[it] = acc;
-                emask |= 1u << it;
+        for (int s = 0; s < 8; ++s) {
+            const bool in = s < nv;
+            r[s] = in ? ld_hint(row + e0 + s, pa) : INT_MAX;
+            c[s] = in ? ld_hint(col + e0 + s, pa) : 0;
+            v[s] = in ? ld_hint(val + e0 + s, pa) : (V)0;
+        }
+    }
+    // rows around the tile (uniform loads)
+    const int rf = __shfl_sync(0xffffffffu, r[0], 0);                       // tile's first row
+    const int before = k0 > 0 ? __ldg(row + k0 - 1) : -1;                  // row before the tile
+    const int64_t nr = k0 + cnt < nnz ? (int64_t)__ldg(row + k0 + cnt) : n_rows;   // next tile's first row
+    const int last_lane = (cnt - 1) >> 3;
+    const int rl = __shfl_sync(0xffffffffu, r[(cnt - 1) & 7], last_lane);   // tile's last row
+    const bool cont = before == rf;                                        // leading continuation
+    const int64_t Wlo = (!ACCUM && t == 0) ? 0 : (int64_t)rf + (cont ? 1 : 0);
+    const int64_t Whi = ACCUM ? (int64_t)rl + 1 : (nr == rl ? nr + 1 : nr);
+    const int64_t L = Whi - Wlo;
+    double yv[kOutQ];
+#pragma unroll
+    for (int q = 0; q < kOutQ; ++q) {
+        const int i = lane + 32 * q;
+        yv[q] = ((ACCUM || !B0) && i < L) ? (double)y[Wlo + i] : 0.0;
+    }
+    if (lane < kOutWin / 32) s_mark[lane] = 0u;
+    double p[8];
+#pragma unroll
+    for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
+    __syncwarp();
+
+    auto emit = [&](int64_t rr, double sum) {
+        const int64_t li = rr - Wlo;
+        if (li >= 0 && li < kOutWin) {
+            s_acc[li] = sum;
+            atomicOr(&s_mark[li >> 5], 1u << (li & 31));
+        } else if (ACCUM) {
+            y[rr] = (V)((double)y[rr] + alpha * sum);
+        } else {
+            y_write<V, B0>(y, rr, sum, alpha, beta);
+        }
+    };
+    int prev = __shfl_up_sync(0xffffffffu, r[7], 1);
+    if (lane == 0) prev = before;
+    double acc = 0.0, head = 0.0;
+    int kseg = 0, cur = -1;
+#pragma unroll
+    for (int s = 0; s < 8; ++s) {
+        if (s < nv) {
+            const int pr = s == 0 ? prev : r[s - 1];
+            if (r[s] != pr) {                                   // a segment (row) starts here
+                if (kseg == 0) head = acc;
+                else emit(cur, acc);                            // closed inside the lane
+                if (!ACCUM && pr >= 0 && (int64_t)r[s] - pr > 1) // empty rows beyond the window
+                    for (int64_t g = max((int64_t)pr + 1, Wlo + kOutWin); g < r[s]; ++g) y_beta<V, B0>(y, g, beta);
+                ++kseg;
+                cur = r[s];
                 acc = 0.0;
-                if (!ACCUM)                                // empty rows beyond the staged window
-                    for (int64_t gq = max((int64_t)r + 1, R0 + kWin); gq < rn; ++gq) y_beta<V, B0>(y, gq, beta);
             }
+            acc += p[s];
         }
     }
-    double incl;
-    const double carry_in = block_seg_scan(emask != 0 || i0 >= cnt, i0 < cnt ? acc : 0.0, &incl);
-    bool first = true;
-#pragma unroll
-    for (int it = 0; it < kIPT; ++it) {
-        if ((emask >> it) & 1u) {
-            const double v = ev[it] + (first ? carry_in : 0.0);
-            first = false;
-            const int64_t r = s_row[i0 + it];
-            const int64_t li = r - R0;
-            if (li < kWin) {
-                s_prod[li] = v;
-                atomicOr(&s_mark[li >> 5], 1u << (li & 31));
-            } else if (ACCUM) {
-                y[r] = (V)((double)y[r] + alpha * v);
-            } else {
-                y_write<V, B0>(y, r, v, alpha, beta);
-            }
-        }
+    if (kseg == 0) head = acc;
+    double Rnext;
+    const double R = seg_suffix(head, kseg > 0 || nv == 0, &Rnext);
+    if (kseg > 0) emit(cur, acc + Rnext);
+    if (lane == 0) {
+        carry_row[t] = cont ? rf : -1;
+        carry_val[t] = cont ? R : 0.0;
     }
-    if (i0 < cnt && i1 == cnt) {                           // CTA carry: the row open at the chunk end
-        const bool open = s_row[cnt] == s_row[cnt - 1];
-        carry_row[blockIdx.x] = open ? s_row[cnt - 1] : -1;
-        carry_val[blockIdx.x] = open ? incl : 0.0;
+    if (!ACCUM && lane == last_lane) {                         // empty rows up to the next tile, beyond the window
+        for (int64_t g = max((int64_t)rl + 1, Wlo + kOutWin); g < nr; ++g) y_beta<V, B0>(y, g, beta);
     }
-    if (!ACCUM && blockIdx.x == 0)                         // leading empty rows beyond the window
-        for (int64_t gq = kWin + threadIdx.x; gq < s_row[0]; gq += kT) y_beta<V, B0>(y, gq, beta);
-    __syncthreads();
+    if (!ACCUM && t == 0)                                      // leading empty rows beyond the window
+        for (int64_t g = kOutWin + lane; g < rf; g += 32) y_beta<V, B0>(y, g, beta);
+    __syncwarp();
 #pragma unroll
-    for (int u = 0; u < kIPT; ++u) {
-        const int i = threadIdx.x + u * kT;
-        if (i < L && i < kWin) {
+    for (int q = 0; q < kOutQ; ++q) {
+        const int i = lane + 32 * q;
+        if (i < L) {
             const bool marked = (s_mark[i >> 5] >> (i & 31)) & 1u;
             if (ACCUM) {
-                if (marked) y[R0 + i] = (V)(yv[u] + alpha * s_prod[i]);
+                if (marked) y[Wlo + i] = (V)(yv[q] + alpha * s_acc[i]);
             } else {
-                double o = marked ? alpha * s_prod[i] : 0.0;
-                if (!B0) o = marked ? fma(beta, yv[u], o) : beta * yv[u];
-                y[R0 + i] = (V)o;
+                double o = marked ? alpha * s_acc[i] : 0.0;
+                if (!B0) o = marked ? fma(beta, yv[q], o) : beta * yv[q];
+                y[Wlo + i] = (V)o;
             }
         }
     }
@@ -354,102 +420,158 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
 
 // ------------------------------------------------------------------ merge-based CSR (K7/G11)
 // "logically partitions the work of processing a group of contiguous
-// rows into equal sized sub-problems".  CTA t consumes merge-path diagonals
-// [t*T, (t+1)*T) of (row ends) x (nonzeros) (coordinates precomputed at conversion,
-// A7).  Row ends and products are staged in shared memory with coalesced loads
-// (all x gathers of the tile in flight at once); y of the tile's rows [r0, r1) is
-// prefetched into registers at the same time.  Each thread consumes kIPT consecutive
-// path items; after the block segmented scan the per-row sums go to shared memory
-// and the tile writes y[r0, r1) coalesced.
+// rows into equal sized sub-problems".  Warp w owns merge-path diagonals
+// [w*T, (w+1)*T) of (row ends) x (nonzeros), T = kMergeItems: rows [r0, r1) end in
+// the tile and nonzeros [k0, k1) are consumed by it (coordinates precomputed at
+// conversion, A7).  Lane l takes the tile's nonzeros [8l, 8l+8): every lane chunk has
+// the same misalignment (k0 mod 4), so the lane loads the covering 16-byte vectors
+// and shifts them by that warp-uniform amount -- products stay in registers with
+// all x gathers in flight.  The tile's row ends (coalesced, shared) mark segment
+// starts in a 256-bit shared bitmap; each lane then reduces its chunk like a CSR5
+// lane (in-lane segments + flag-segmented suffix sum over lanes).  Every row ending
+// in the tile is written by it (empty rows: beta*y); row r0 may have begun in an
+// earlier tile (its earlier parts arrive as carries); the part of row r1 inside the
+// tile is the tile carry.  The row window is written back coalesced.
+template <typename V> struct ShiftLoad8;
+template <> struct ShiftLoad8<double> {    // 8 doubles from p (8-byte aligned): 5 x double2, shift 0/1
+    static __device__ __forceinline__ void load(const double *p, double (&v)[8], uint64_t pol) {
+        const int m = (int)(((uintptr_t)p >> 3) & 1);
+        const double2 *b = reinterpret_cast<const double2 *>(p - m);
+        double w[10];
+#pragma unroll
+        for (int q = 0; q < 5; ++q) { double2 t = ld_hint(b + q, pol); w[2 * q] = t.x; w[2 * q + 1] = t.y; }
+#pragma unroll
+        for (int s = 0; s < 8; ++s) v[s] = m ? w[s + 1] : w[s];
+    }
+};
+template <> struct ShiftLoad8<float> {     // 8 floats: 3 x float4, shift 0..3
+    static __device__ __forceinline__ void load(const float *p, float (&v)[8], uint64_t pol) {
+        const int m = (int)(((uintptr_t)p >> 2) & 3);
+        const float4 *b = reinterpret_cast<const float4 *>(p - m);
+        float w[12];
+#pragma unroll
+        for (int q = 0; q < 3; ++q) { float4 t = ld_hint(b + q, pol); w[4*q] = t.x; w[4*q+1] = t.y; w[4*q+2] = t.z; w[4*q+3] = t.w; }
+#pragma unroll
+        for (int s = 0; s < 8; ++s) v[s] = m == 0 ? w[s] : m == 1 ? w[s + 1] : m == 2 ? w[s + 2] : w[s + 3];
+    }
+};
+__device__ __forceinline__ void shift_load_int8(const int *p, int (&v)[8], uint64_t pol) {
+    const int m = (int)(((uintptr_t)p >> 2) & 3);
+    const int4 *b = reinterpret_cast<const int4 *>(p - m);
+    int w[12];
+#pragma unroll
+    for (int q = 0; q < 3; ++q) { int4 t = ld_hint(b + q, pol); w[4*q] = t.x; w[4*q+1] = t.y; w[4*q+2] = t.z; w[4*q+3] = t.w; }
+#pragma unroll
+    for (int s = 0; s < 8; ++s) v[s] = m == 0 ? w[s] : m == 1 ? w[s + 1] : m == 2 ? w[s + 2] : w[s + 3];
+}
+
 template <typename V, typename IT, bool B0>
-__global__ void __launch_bounds__(kT)
+__global__ void __launch_bounds__(kT, kMinBlocks)
 k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
-        const int64_t *__restrict__ crow, const int64_t *__restrict__ cnz, int64_t n_rows,
+        const int64_t *__restrict__ crow, const int64_t *__restrict__ cnz, int64_t n_tiles, int64_t n_rows,
         const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
         int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
-    __shared__ int s_end[kMergeItems];
-    __shared__ double s_prod[kMergeItems];          // products, then per-row sums
+    constexpr int TI = (int)kMergeItems;
+    static_assert(TI == 256 && kWIPT == 8, "merge tile is 32 lanes x 8");
+    __shared__ double s_sum_all[kT / 32][TI];             // row sums (local row index)
+    __shared__ int s_end_all[kT / 32][TI];                // local end of local row i
+    __shared__ unsigned short s_rowat_all[kT / 32][TI];   // local row starting at a position
+    __shared__ unsigned s_flag_all[kT / 32][TI / 32];
+    __shared__ unsigned s_mark_all[kT / 32][TI / 32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    if (t >= n_tiles) return;
+    double *s_sum = s_sum_all[wid];
+    int *s_end = s_end_all[wid];
+    unsigned short *s_rowat = s_rowat_all[wid];
+    unsigned *s_flag = s_flag_all[wid];
+    unsigned *s_mark = s_mark_all[wid];
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
-    const int64_t t = blockIdx.x;
-    const int64_t r0 = crow[t], k0 = cnz[t], r1 = crow[t + 1], k1 = cnz[t + 1];
-    const int nrows = (int)(r1 - r0), nnzt = (int)(k1 - k0), items = nrows + nnzt;
-    double yv[kIPT];
-#pragma unroll
-    for (int u = 0; u < kIPT; ++u) {
-        const int i = threadIdx.x + u * kT;
-        yv[u] = (!B0 && i < nrows) ? (double)y[r0 + i] : 0.0;
+    const int64_t r0 = __ldg(crow + t), k0 = __ldg(cnz + t), r1 = __ldg(crow + t + 1), k1 = __ldg(cnz + t + 1);
+    const int nrows = (int)(r1 - r0), nnzt = (int)(k1 - k0);
+    const int j0 = lane * 8;
+    const int nv = max(0, min(8, nnzt - j0));
+    int c[8];
+    V v[8];
+    if (nv > 0) {
+        shift_load_int8(col + k0 + j0, c, pa);
+        ShiftLoad8<V>::load(val + k0 + j0, v, pa);
     }
+    double yv[kOutQ];
 #pragma unroll
-    for (int u = 0; u < kIPT; ++u) {
-        const int i = threadIdx.x + u * kT;
-        if (i < nrows) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
+    for (int q = 0; q < kOutQ; ++q) {
+        const int i = lane + 32 * q;
+        yv[q] = (!B0 && i < nrows) ? (double)y[r0 + i] : 0.0;
     }
+    for (int i = lane; i < nrows; i += 32) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
+    const bool r0_inside = (int64_t)__ldg(rp + r0) == k0;   // A7: rp[r0] <= k0 always
+    if (lane < TI / 32) { s_flag[lane] = 0u; s_mark[lane] = 0u; }
+    double p[8];
 #pragma unroll
-    for (int u = 0; u < kIPT; ++u) {
-        const int j = threadIdx.x + u * kT;
-        if (j < nnzt) {
-            const int c = ld_hint(col + k0 + j, pa);
-            const V v = ld_hint(val + k0 + j, pa);
-            s_prod[j] = (double)v * (double)ld_x(x + c, px);
+    for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
+    __syncwarp();
+    // segment starts: local row i (1 <= i <= nrows) starts at s_end[i-1]; row 0 at 0 if r0_inside
+    for (int i = lane; i <= nrows; i += 32) {
+        const int st = i == 0 ? 0 : s_end[i - 1];
+        const int en = i < nrows ? s_end[i] : nnzt;         // open row r1 runs past the tile
+        if ((i > 0 || r0_inside) && st < nnzt && en > st) {
+            atomicOr(&s_flag[st >> 5], 1u << (st & 31));
+            s_rowat[st] = (unsigned short)i;
         }
     }
-    __syncthreads();
-    // this thread's start on the tile's merge path: largest i with s_end[i-1] + i <= d
-    const int d = threadIdx.x * kIPT;
-    const int nit = max(0, min(kIPT, items - d));
-    int lo = max(0, d - nnzt), hi = min(d, nrows);
-    while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (s_end[mid - 1] + mid <= d) lo = mid; else hi = mid - 1;
-    }
-    int i = lo, j = d - lo;
-    const int first_local = i;
-    unsigned emask = 0;
-    double ev[kIPT];
-    double acc = 0.0;
+    __syncwarp();
+    const unsigned fl = nv > 0 ? ((s_flag[j0 >> 5] >> (j0 & 31)) & 0xFFu) : 0u;
+    auto put = [&](int li, double sum) {
+        s_sum[li] = sum;
+        atomicOr(&s_mark[li >> 5], 1u << (li & 31));
+    };
+    double acc = 0.0, head = 0.0;
+    int kseg = 0, cur = -1;
 #pragma unroll
-    for (int it = 0; it < kIPT; ++it) {
-        ev[it] = 0.0;
-        if (it < nit) {
-            if (i < nrows && s_end[i] <= j) {              // row r0+i ends (A7 tie-break)
-                ev[it] = acc;
-                emask |= 1u << it;
-                acc = 0.0;
-                ++i;
-            } else {
-                acc += s_prod[j];
-                ++j;
-            }
+    for (int s = 0; s < 8; ++s) {
+        if ((fl >> s) & 1u) {
+            if (kseg == 0) head = acc;
+            else put(cur, acc);                           // closed inside the lane (cur < nrows)
+            ++kseg;
+            cur = s_rowat[j0 + s];
+            acc = 0.0;
+        }
+        acc += p[s];
+    }
+    if (kseg == 0) head = acc;
+    double Rnext;
+    const double R = seg_suffix(head, kseg > 0 || nv == 0, &Rnext);
+    const double lead = __shfl_sync(0xffffffffu, R, 0);  // nonzeros before the tile's first segment
+    double cv = 0.0;
+    int cset = 0;
+    if (kseg > 0) {
+        const double tot = acc + Rnext;
+        if (cur < nrows) put(cur, tot);
+        else { cv = tot; cset = 1; }                      // row r1 started in this tile
+    }
+    if (lane == 0 && !r0_inside && nnzt > 0) {
+        if (nrows > 0) put(0, lead);                      // row r0 ends here
+        else { cv = lead; cset = 1; }                     // the tile is the middle of row r0 == r1
+    }
+    const unsigned who = __ballot_sync(0xffffffffu, cset);
+    if (lane == 0 && who == 0) { carry_row[t] = -1; carry_val[t] = 0.0; }
+    if (cset) { carry_row[t] = r1; carry_val[t] = cv; }
+    __syncwarp();
+#pragma unroll
+    for (int q = 0; q < kOutQ; ++q) {
+        const int i = lane + 32 * q;
+        if (i < nrows) {
+            const bool marked = (s_mark[i >> 5] >> (i & 31)) & 1u;
+            double o = marked ? alpha * s_sum[i] : 0.0;
+            if (!B0) o = fma(beta, yv[q], o);
+            y[r0 + i] = (V)o;
         }
     }
-    double incl;
-    const double carry_in = block_seg_scan(emask != 0 || nit == 0, nit ? acc : 0.0, &incl);
-    // (the scan's barriers guarantee every walk is done: s_prod is free for row sums)
-    int li = first_local;
-    bool first = true;
-#pragma unroll
-    for (int it = 0; it < kIPT; ++it) {
-        if ((emask >> it) & 1u) {
-            s_prod[li] = ev[it] + (first ? carry_in : 0.0);
-            first = false;
-            ++li;
-        }
-    }
-    // tile carry: nonzeros after the tile's last row end belong to row r1 (ends later)
-    if (nit > 0 && d + nit == items) {
-        const bool open = r1 < n_rows && k1 > (nrows ? k0 + s_end[nrows - 1] : k0);
-        carry_row[t] = open ? r1 : -1;
-        carry_val[t] = open ? incl : 0.0;
-    }
-    __syncthreads();
-#pragma unroll
-    for (int u = 0; u < kIPT; ++u) {
-        const int q = threadIdx.x + u * kT;
-        if (q < nrows) {
-            double o = alpha * s_prod[q];
-            if (!B0) o = fma(beta, yv[u], o);
-            y[r0 + q] = (V)o;
-        }
+    for (int i = kOutWin + lane; i < nrows; i += 32) {        // rows beyond the prefetched window
+        const bool marked = (s_mark[i >> 5] >> (i & 31)) & 1u;
+        double o = marked ? alpha * s_sum[i] : 0.0;
+        if (!B0) o = fma(beta, (double)y[r0 + i], o);
+        y[r0 + i] = (V)o;
     }
 }
 
@@ -704,23 +826,23 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
             x, y, n, alpha, beta);
         SPMV_LAUNCH_CHECK();
         if (h->hyb_coo_nnz == 0) return SPMV_OK;
-        k_coo<V, true, B0><<<(unsigned)h->n_carry, kT, 0, s>>>(
+        k_coo<V, true, B0><<<(unsigned)ceil_div<int64_t>(h->n_carry, kT / 32), kT, 0, s>>>(
             (const int *)h->arr[SPMV_ARR_COO_ROW].p, (const int *)h->arr[SPMV_ARR_HYB_COO_COL].p,
-            (const V *)h->arr[SPMV_ARR_HYB_COO_VAL].p, h->hyb_coo_nnz, x, y, n, alpha, beta, crow, cval);
+            (const V *)h->arr[SPMV_ARR_HYB_COO_VAL].p, h->hyb_coo_nnz, h->n_carry, x, y, n, alpha, beta, crow, cval);
         SPMV_LAUNCH_CHECK();
         return launch_fixup<V>(h, y, alpha, s);
     }
     case SPMV_COO:
         if (h->nnz == 0) return launch_scale<V, B0>(h, y, beta, s);
-        k_coo<V, false, B0><<<(unsigned)h->n_carry, kT, 0, s>>>(
-            (const int *)h->arr[SPMV_ARR_COO_ROW].p, col, val, h->nnz, x, y, n, alpha, beta, crow, cval);
+        k_coo<V, false, B0><<<(unsigned)ceil_div<int64_t>(h->n_carry, kT / 32), kT, 0, s>>>(
+            (const int *)h->arr[SPMV_ARR_COO_ROW].p, col, val, h->nnz, h->n_carry, x, y, n, alpha, beta, crow, cval);
         SPMV_LAUNCH_CHECK();
         return launch_fixup<V>(h, y, alpha, s);
     case SPMV_MERGE:
         if (h->merge_tiles == 0) return SPMV_OK;
-        k_merge<V, IT, B0><<<(unsigned)h->merge_tiles, kT, 0, s>>>(
+        k_merge<V, IT, B0><<<(unsigned)ceil_div<int64_t>(h->merge_tiles, kT / 32), kT, 0, s>>>(
             rp, col, val, (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_ROW].p,
-            (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_NZ].p, n, x, y, alpha, beta, crow, cval);
+            (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_NZ].p, h->merge_tiles, n, x, y, alpha, beta, crow, cval);
         SPMV_LAUNCH_CHECK();
         return launch_fixup<V>(h, y, alpha, s);
     case SPMV_CSR5: {
