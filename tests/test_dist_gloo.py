@@ -1,0 +1,95 @@
+"""Multi-process logic of the row-partitioned SpMV on CPU (gloo, world size 2 and 3),
+SURVEY §4 T4': partition + remap + padded slots + all-gather of x + a per-shard SpMV,
+compared with the unpartitioned product.  The per-shard SpMV here is the ORACLE (test
+harness only); the GPU path runs the same ShardLayout / all_gather_slots plumbing with
+libspmv shards (bench.py --gpus N, tests/test_gpu_dist.py)."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import matgen
+import oracle
+from paper_conf_ipps_nisassvs18_b200.dist import ShardLayout, all_gather_slots
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, case, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        if case == "rmat":
+            A = matgen.rmat(11, seed=31)
+        elif case == "lap":
+            A = matgen.laplacian5(40)
+        else:                                    # empty rows and a long row
+            lens = np.random.default_rng(5).integers(0, 7, 3000)
+            lens[100:400] = 0
+            lens[2000] = 2500
+            A = matgen.from_lengths(lens, 3000, seed=33)
+        x = matgen.vector(A.n_cols, 32, 1)
+        y = matgen.vector(A.n_rows, 32, 2)
+        splits = oracle.partition(A, world)
+        lay = ShardLayout(splits, rank)
+        # every rank holds only its x slice; the gathered vector is built by the collective
+        slot = lay.pack_x(torch.from_numpy(x[lay.r0:lay.r1].copy()))
+        gathered = torch.zeros(world * lay.S, dtype=torch.float64)
+        all_gather_slots(gathered, slot)
+        rp, col, val = oracle.slice_remap(A, splits, rank)
+        shard = matgen.HostCSR(rp, col, val, lay.rows, world * lay.S)
+        y_local = oracle.spmv_csr(shard, gathered.numpy(), 1.25, -0.5, y[lay.r0:lay.r1])
+        # slot_of agrees with the remap
+        for k in range(0, A.nnz, max(1, A.nnz // 50)):
+            r = int(np.searchsorted(A.row_ptr, k, side="right")) - 1
+            if lay.r0 <= r < lay.r1:
+                assert col[k - A.row_ptr[lay.r0]] == lay.slot_of(int(A.col[k]))
+        # assemble y for the check (padded equal-count gather)
+        yslot = lay.pack_x(torch.from_numpy(y_local))
+        yall = torch.zeros(world * lay.S, dtype=torch.float64)
+        all_gather_slots(yall, yslot)
+        if rank == 0:
+            full = np.concatenate([yall[k * lay.S: k * lay.S + int(splits[k + 1] - splits[k])].numpy()
+                                   for k in range(world)])
+            ref = oracle.spmv_csr(A, x, 1.25, -0.5, y)
+            q.put(bool(np.array_equal(full, ref)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+@pytest.mark.parametrize("case", ["rmat", "lap", "ragged"])
+def test_partitioned_spmv_gloo(world, case):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, case, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(120)
+        assert p.exitcode == 0
+    assert q.get(timeout=10) is True
+
+
+def test_layout_host_logic():
+    splits = np.array([0, 3, 3, 10], dtype=np.int64)     # an empty middle part
+    lay = ShardLayout(splits, 2)
+    assert (lay.P, lay.S, lay.r0, lay.r1, lay.rows) == (3, 7, 3, 10, 7)
+    assert lay.slot_of(0) == 0 and lay.slot_of(2) == 2
+    assert lay.slot_of(3) == 2 * 7 + 0 and lay.slot_of(9) == 2 * 7 + 6
+    v = lay.pack_x(torch.arange(7, dtype=torch.float64))
+    assert v.tolist() == list(range(7))
+    lay0 = ShardLayout(splits, 0)
+    assert lay0.pack_x(torch.ones(3, dtype=torch.float64)).tolist() == [1, 1, 1, 0, 0, 0, 0]
