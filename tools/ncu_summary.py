@@ -1,0 +1,153 @@
+"""Summarise ncu outputs into tracked profiles/ files.
+
+  python tools/ncu_summary.py launches  <launches.csv> <out.md>
+  python tools/ncu_summary.py full      <report.ncu-rep> <out.md> [--traffic CONFIG DTYPE]
+
+`launches` aggregates a `--metrics gpu__time_duration.sum` launch list per kernel
+(count, mean, total, share).  `full` prints, per captured launch, duration, DRAM
+bytes / throughput, L1/L2 hit rates, occupancy, registers and the top stall reasons;
+with --traffic it also records DRAM bytes per launch of each format's SpMV kernel in
+profiles/ncu_traffic.json (read by bench.py's roofline.traffic).
+"""
+import collections
+import csv
+import io
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def short(name):
+    n = name.split("(")[0].replace("void ", "").replace("(anonymous namespace)::", "")
+    n = n.replace("spmv::<unnamed>::", "").replace("<unnamed>::", "").strip()
+    i = n.find("k_")
+    if n.startswith("unnamed>::") or (i > 0 and "::" in n[:i]):
+        n = n[i:]
+    return n
+
+
+def launches(path, out):
+    rows = list(csv.reader(open(path)))
+    i = [k for k, r in enumerate(rows) if "Kernel Name" in r][0]
+    hdr = rows[i]
+    agg = collections.OrderedDict()
+    for r in rows[i + 1:]:
+        d = dict(zip(hdr, r))
+        if d.get("Metric Name") != "gpu__time_duration.sum":
+            continue
+        v = float(d["Metric Value"].replace(",", ""))
+        unit = d["Metric Unit"]
+        us = v / 1000 if unit == "ns" else (v * 1000 if unit == "ms" else v)
+        agg.setdefault(short(d["Kernel Name"]), []).append(us)
+    spmv = {k: v for k, v in agg.items() if k.startswith("k_")}
+    tot = sum(sum(v) for v in spmv.values())
+    with open(out, "w") as f:
+        f.write(f"# ncu launch list summary: {os.path.basename(path)}\n\n")
+        f.write("ncu --metrics gpu__time_duration.sum --clock-control none (serialised, cold-cache: compare "
+                "shares, not absolutes)\n\n")
+        f.write("| kernel | launches | mean us | total us | share of libspmv time |\n|---|---|---|---|---|\n")
+        for k, v in agg.items():
+            s = sum(v)
+            share = f"{100 * s / tot:.1f}%" if k in spmv and tot else "-"
+            f.write(f"| `{k}` | {len(v)} | {s / len(v):.1f} | {s:.1f} | {share} |\n")
+        # share of one timed step: the step's SpMV launches (beta != 0 variants, fix-ups)
+        step = {k: sum(v) / len(v) * (2 if k.startswith("k_ell<") and "1>" not in k else 1)
+                for k, v in agg.items()
+                if k.split("<")[0] in ("k_coo", "k_ell", "k_csr_vector", "k_merge", "k_csr5") and not k.endswith("1>")}
+        fix = agg.get("k_fixup<double>") or agg.get("k_fixup<float>")
+        if fix:
+            step["k_fixup (x launches per step)"] = sum(fix) / len(fix) * 3
+        st = sum(step.values())
+        f.write("\n## Share of one bench step (mean launch time x launches per step)\n\n")
+        f.write("| kernel | us per step | share |\n|---|---|---|\n")
+        for k, v in sorted(step.items(), key=lambda kv: -kv[1]):
+            f.write(f"| `{k}` | {v:.1f} | {100 * v / st:.1f}% |\n")
+    print(open(out).read())
+
+
+KEYS = [
+    ("gpu__time_duration.sum", "time"),
+    ("dram__bytes_read.sum", "dram_rd"),
+    ("dram__bytes_write.sum", "dram_wr"),
+    ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "dram%"),
+    ("lts__t_sector_hit_rate.pct", "L2hit%"),
+    ("l1tex__t_sector_hit_rate.pct", "L1hit%"),
+    ("l1tex__throughput.avg.pct_of_peak_sustained_elapsed", "L1thr%"),
+    ("sm__warps_active.avg.pct_of_peak_sustained_active", "warps%"),
+    ("launch__registers_per_thread", "regs"),
+    ("smsp__inst_executed.sum", "warp_inst"),
+]
+
+
+def to_bytes(v, unit):
+    m = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
+    return float(v.replace(",", "")) * m.get(unit, 1)
+
+
+def full(rep, out, traffic=None, formats=("coo", "ell", "csr", "hyb", "merge", "csr5")):
+    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    r = list(csv.reader(io.StringIO(raw)))
+    hdr, units = r[0], r[1]
+    pre = "smsp__average_warps_issue_stalled_"
+    lines = [f"# ncu --set full summary: {os.path.basename(rep)}\n",
+             "ncu --set full --clock-control none --import-source on (one replayed launch per row)\n",
+             "| kernel | " + " | ".join(k[1] for k in KEYS) + " | top stalls (warps per issue) |",
+             "|---|" + "---|" * (len(KEYS) + 1)]
+    seen = collections.Counter()
+    trafficmap = {}
+    for row in r[2:]:
+        d = dict(zip(hdr, row))
+        name = short(d["Kernel Name"])
+        cells = []
+        for k, _ in KEYS:
+            u = units[hdr.index(k)] if k in hdr else ""
+            cells.append(f"{d.get(k, '')} {u}".strip())
+        st = {h[len(pre):].replace("_per_issue_active.ratio", ""): float(d[h]) for h in hdr
+              if h.startswith(pre) and h.endswith("_per_issue_active.ratio") and d[h] not in ("", "n/a")}
+        top = ", ".join(f"{k} {v:.1f}" for v, k in sorted(((v, k) for k, v in st.items()), reverse=True)[:3])
+        lines.append(f"| `{name}` | " + " | ".join(cells) + f" | {top} |")
+        base = name.split("<")[0]
+        seen[base] += 1
+        targs = name.split("<")[1] if "<" in name else ""
+        fmt = {"k_merge": "merge", "k_csr5": "csr5"}.get(base)
+        if base == "k_coo":
+            fmt = "hyb" if targs.split(",")[1].strip() in ("1", "true") else "coo"
+        elif base == "k_ell":
+            fmt = "ell" if ("ell" in formats and seen[base] == 1) else "hyb"
+        elif base == "k_csr_vector" and seen[base] == 1 and "csr" in formats:
+            fmt = "csr"
+        if fmt:
+            rd = to_bytes(d["dram__bytes_read.sum"], units[hdr.index("dram__bytes_read.sum")])
+            wr = to_bytes(d["dram__bytes_write.sum"], units[hdr.index("dram__bytes_write.sum")])
+            if fmt == "hyb" or fmt not in trafficmap:
+                trafficmap[fmt] = trafficmap.get(fmt, 0) + rd + wr
+    with open(out, "w") as f:
+        f.write("\n".join(lines) + "\n")
+    print("\n".join(lines))
+    if traffic:
+        cfg, dt = traffic
+        p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+        d = json.load(open(p)) if os.path.exists(p) else {}
+        d.setdefault(cfg, {}).setdefault(dt, {}).update({k: int(v) for k, v in trafficmap.items()})
+        d["_note"] = ("DRAM bytes (read+write) per launch of each format's SpMV kernel, from one ncu --set full "
+                      "capture of the bench command's consistency probe (alpha=beta=1); see profiles/*.md")
+        json.dump(d, open(p, "w"), indent=1, sort_keys=True)
+        print("traffic:", trafficmap)
+
+
+if __name__ == "__main__":
+    mode = sys.argv[1]
+    if mode == "launches":
+        launches(sys.argv[2], sys.argv[3])
+    else:
+        tr = None
+        if "--traffic" in sys.argv:
+            i = sys.argv.index("--traffic")
+            tr = (sys.argv[i + 1], sys.argv[i + 2])
+        fm = ("coo", "ell", "csr", "hyb", "merge", "csr5")
+        if "--formats" in sys.argv:
+            fm = tuple(sys.argv[sys.argv.index("--formats") + 1].split(","))
+        full(sys.argv[2], sys.argv[3], tr, fm)
