@@ -200,3 +200,93 @@ def from_rows(rows, n_cols) -> HostCSR:
         row_ptr.append(len(col))
     return HostCSR(np.array(row_ptr, dtype=np.int64), np.array(col, dtype=np.int32),
                    np.array(val, dtype=np.float64), len(rows), int(n_cols), "rows")
+
+
+# ----------------------------------------------------------------------------- cfg4 sweep
+
+#: Table I nnz buckets: (lo, hi, count of 2299); upper bound 96M
+NNZ_BUCKETS = [(3, 10_000, 747), (10_000, 50_000, 508), (50_000, 100_000, 209), (100_000, 500_000, 362),
+               (500_000, 1_000_000, 147), (1_000_000, 5_000_000, 208), (5_000_000, 50_000_000, 109),
+               (50_000_000, 96_000_000, 9)]
+FAMILIES = ("uniform", "banded", "blockdiag", "powerlaw", "mixed")
+
+
+def _loguniform(rng, lo, hi):
+    return float(np.exp(rng.uniform(np.log(lo), np.log(hi))))
+
+
+def sweep_params(i, max_nnz=None):
+    """Parameters of sweep matrix i: family = i mod 5,
+    nnz bucket drawn with Table I frequencies, log-uniform within it; mu log-uniform in
+    [1, 256]; n_rows = max(8, nnz/mu); 80% square, else aspect log-uniform in [1/4, 4]."""
+    rng = np.random.default_rng(SEEDS["sweep"] + i)
+    fam = FAMILIES[i % 5]
+    w = np.array([b[2] for b in NNZ_BUCKETS], dtype=float)
+    b = NNZ_BUCKETS[int(rng.choice(len(NNZ_BUCKETS), p=w / w.sum()))]
+    nnz = int(_loguniform(rng, b[0], b[1]))
+    if max_nnz:
+        nnz = min(nnz, int(max_nnz))
+    mu = _loguniform(rng, 1.0, 256.0)
+    n_rows = max(8, int(nnz / mu))
+    aspect = 1.0 if rng.random() < 0.8 else _loguniform(rng, 0.25, 4.0)
+    n_cols = max(8, int(n_rows * aspect))
+    p = dict(i=i, family=fam, nnz_target=nnz, mu=mu, n_rows=n_rows, n_cols=n_cols, seed=SEEDS["sweep"] + i)
+    if fam == "banded":
+        p["fill"] = float(rng.uniform(0.3, 1.0))
+    elif fam == "blockdiag":
+        p["block"] = int(_loguniform(rng, 4, 256))
+        p["fill"] = float(rng.uniform(0.3, 1.0))
+        p["noise"] = float(rng.uniform(0.0, 0.05))
+        # rows of a block hold ~block*fill entries: size the matrix to the nnz target
+        p["n_rows"] = max(8, int(nnz / (p["block"] * p["fill"])))
+        p["n_cols"] = max(8, int(p["n_rows"] * aspect))
+    elif fam == "powerlaw":
+        p["gamma"] = float(rng.uniform(1.5, 3.0))
+    elif fam == "mixed":
+        p["q"] = float(_loguniform(rng, 0.005, 0.10))
+        p["long"] = float(rng.uniform(10.0, 100.0))
+    return p
+
+
+def _union_rows(A: HostCSR, B: HostCSR) -> HostCSR:
+    """Row-wise union of two structures (duplicates coalesced; A's values kept)."""
+    ra = np.repeat(np.arange(A.n_rows, dtype=np.int64), np.diff(A.row_ptr))
+    rb = np.repeat(np.arange(B.n_rows, dtype=np.int64), np.diff(B.row_ptr))
+    keys = np.concatenate([ra * A.n_cols + A.col, rb * A.n_cols + B.col])
+    keys = np.unique(keys)
+    rows = keys // A.n_cols
+    row_ptr = np.zeros(A.n_rows + 1, dtype=np.int64)
+    np.add.at(row_ptr, rows + 1, 1)
+    np.cumsum(row_ptr, out=row_ptr)
+    return HostCSR(row_ptr, (keys % A.n_cols).astype(np.int32), np.empty(0), A.n_rows, A.n_cols, A.name)
+
+
+def sweep_matrix(i, kind="f64", max_nnz=None):
+    """Build sweep matrix i (canonical CSR, seeded values).  Returns (HostCSR, params)."""
+    p = sweep_params(i, max_nnz)
+    rng = np.random.default_rng(p["seed"] + 1)
+    n, m, mu, seed = p["n_rows"], p["n_cols"], p["mu"], p["seed"]
+    fam = p["family"]
+    if fam == "uniform":
+        lens = np.minimum(rng.poisson(mu, n), m)
+        A = from_lengths(lens, m, seed, kind)
+    elif fam == "banded":
+        half = max(0, int(round(mu / (2 * p["fill"]) - 0.5)))
+        A = window(n, m, half, p["fill"], seed, 0, kind)
+    elif fam == "blockdiag":
+        bsz = min(p["block"], n)
+        base = window(n, m, bsz, p["fill"], seed, 1, "ones")
+        nl = np.minimum(rng.poisson(p["noise"] * max(1.0, base.nnz / n), n), m)
+        noise = from_lengths(nl, m, seed + 3, "ones")
+        A = set_values(_union_rows(base, noise), seed + 5, kind)
+    elif fam == "powerlaw":
+        raw = rng.pareto(p["gamma"] - 1.0, n) + 1.0
+        lens = np.minimum(np.maximum(0, np.round(raw * mu / raw.mean())), m).astype(np.int64)
+        A = from_lengths(lens, m, seed, kind)
+    else:  # mixed
+        lens = rng.poisson(mu, n)
+        long = rng.random(n) < p["q"]
+        lens[long] = (mu * rng.uniform(10.0, p["long"], long.sum())).astype(np.int64)
+        A = from_lengths(np.minimum(lens, m), m, seed, kind)
+    A.name = f"sweep{i}-{fam}"
+    return A, p

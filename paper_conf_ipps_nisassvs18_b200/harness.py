@@ -76,7 +76,9 @@ def measure_matrix(A: CSR, formats: Iterable[str] = PAPER_FORMATS, reps: int = 5
                    x: Optional[torch.Tensor] = None, y: Optional[torch.Tensor] = None,
                    **convert_opts) -> Dict[str, object]:
     """Convert A to each format, time it, and emit the per-format record + labels
-    (the paper's ground truth, regenerated on this GPU)."""
+    (the paper's ground truth, regenerated on this GPU).  Before timing, every format's
+    y = A x + y0 is compared with the CSR result (max |diff| / (max |y| + 1) recorded
+    as "agree"); the oracle parity of each kernel is established by tests/, not here."""
     dev = A.row_ptr.device
     if x is None:
         x = torch.ones(A.n_cols, dtype=A.dtype, device=dev)
@@ -84,6 +86,7 @@ def measure_matrix(A: CSR, formats: Iterable[str] = PAPER_FORMATS, reps: int = 5
         y = torch.zeros(A.n_rows, dtype=A.dtype, device=dev)
     rec: Dict[str, object] = {"formats": {}}
     times: Dict[str, Optional[float]] = {}
+    ref_y = None
     for f in formats:
         try:
             h = convert(A, f, **convert_opts)
@@ -93,16 +96,71 @@ def measure_matrix(A: CSR, formats: Iterable[str] = PAPER_FORMATS, reps: int = 5
                 times[f] = None
                 continue
             raise
+        yc = y.clone()
+        h.run(1.0, x, 1.0, yc)
+        if ref_y is None:
+            ref_y = yc
+        agree = float((yc - ref_y).abs().max().item() / (ref_y.abs().max().item() + 1.0)) if A.n_rows else 0.0
         t = time_handle(h, x, y, reps=reps, warmup=warmup)
         info = h.info()
         gflops = 2.0 * A.nnz / (t["t_mean_ms"] * 1e-3) / 1e9 if t["t_mean_ms"] > 0 else 0.0
         gbs = info["bytes_per_run"] / (t["t_mean_ms"] * 1e-3) / 1e9 if t["t_mean_ms"] > 0 else 0.0
         rec["formats"][f] = {**t, "gflops": gflops, "gbs_own": gbs, "bytes_per_run": info["bytes_per_run"],
-                             "launches": h.launches()}
+                             "launches": h.launches(), "agree": agree}
         times[f] = t["t_mean_ms"]
         h.destroy()
     rec.update(labels(times))
     return rec
+
+
+def sweep(start: int = 0, count: int = 2000, out: str = "sweep.jsonl", dtype: str = "f64", reps: int = 50,
+          warmup: int = 5, shard: int = 0, nshards: int = 1, max_nnz: Optional[int] = None) -> int:
+    """BASELINE configs[3]: the format-selection sweep.  Matrices start..start+count-1
+    (matgen.sweep_matrix, seeded), this process takes i % nshards == shard (replicas over
+    GPUs).  One JSONL record per matrix: generator parameters, the 17 features + extras
+    (spmv_features), per-format timings and labels.  Resumable: ids already in `out`
+    are skipped.  Returns the number of matrices measured."""
+    import json
+    import os
+    import time
+
+    import matgen
+
+    from .spmv import PAPER_FEATURES, features
+
+    done = set()
+    if os.path.exists(out):
+        with open(out) as fh:
+            for line in fh:
+                try:
+                    done.add(json.loads(line)["i"])
+                except Exception:
+                    pass
+    tdt = torch.float64 if dtype == "f64" else torch.float32
+    n = 0
+    with open(out, "a") as fh:
+        for i in range(start, start + count):
+            if i % nshards != shard or i in done:
+                continue
+            t0 = time.time()
+            A, p = matgen.sweep_matrix(i, dtype, max_nnz)
+            dA = CSR.from_host(A, dtype=tdt)
+            feats = features(dA)
+            x = torch.from_numpy(matgen.vector(A.n_cols, p["seed"], 1, dtype)).to(dA.row_ptr.device).to(tdt)
+            y = torch.from_numpy(matgen.vector(A.n_rows, p["seed"], 2, dtype)).to(dA.row_ptr.device).to(tdt)
+            rec = measure_matrix(dA, reps=reps, warmup=warmup, x=x, y=y)
+            row = {"i": i, "params": p, "dtype": dtype, "n_rows": A.n_rows, "n_cols": A.n_cols, "nnz": A.nnz,
+                   "features": {k: feats[k] for k in PAPER_FEATURES},
+                   "extras": {k: feats[k] for k in ("ell_width", "ell_slots", "ell_pad_frac", "hyb_width",
+                                                      "hyb_coo_nnz", "hyb_width_floor", "hyb_width_cusp",
+                                                      "n_empty_rows")},
+                   "gpu": torch.cuda.get_device_name(), "wall_s": None, **rec}
+            row["wall_s"] = round(time.time() - t0, 3)
+            fh.write(json.dumps(row) + "\n")
+            fh.flush()
+            n += 1
+            del dA
+    return n
 
 
 def best_format(rec: Dict[str, object]) -> Optional[str]:
@@ -112,3 +170,27 @@ def best_format(rec: Dict[str, object]) -> Optional[str]:
 def records_to_rows(recs: List[Dict[str, object]]) -> List[Dict[str, object]]:
     """Flatten measure_matrix records (one JSONL line per matrix)."""
     return [dict(r) for r in recs]
+
+
+def _main():
+    import argparse
+    ap = argparse.ArgumentParser(description="format-selection sweep (BASELINE configs[3])")
+    ap.add_argument("--start", type=int, default=0)
+    ap.add_argument("--count", type=int, default=2000)
+    ap.add_argument("--out", default="sweep.jsonl")
+    ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
+    ap.add_argument("--reps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--max-nnz", type=int, default=None)
+    a = ap.parse_args()
+    import os
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
+    out = a.out if ws == 1 else a.out.replace(".jsonl", f".rank{rank}.jsonl")
+    n = sweep(a.start, a.count, out, a.dtype, a.reps, a.warmup, rank, ws, a.max_nnz)
+    print(f"rank {rank}: measured {n} matrices -> {out}")
+
+
+if __name__ == "__main__":
+    _main()
