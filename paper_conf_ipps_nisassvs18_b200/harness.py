@@ -101,7 +101,7 @@ def measure_matrix(A: CSR, formats: Iterable[str] = PAPER_FORMATS, reps: int = 5
         if ref_y is None:
             ref_y = yc
         agree = float((yc - ref_y).abs().max().item() / (ref_y.abs().max().item() + 1.0)) if A.n_rows else 0.0
-        t = time_handle(h, x, y, reps=reps, warmup=warmup)
+        t = time_handle(h, x, y.clone(), reps=reps, warmup=warmup)   # timing accumulates into a scratch y
         info = h.info()
         gflops = 2.0 * A.nnz / (t["t_mean_ms"] * 1e-3) / 1e9 if t["t_mean_ms"] > 0 else 0.0
         gbs = info["bytes_per_run"] / (t["t_mean_ms"] * 1e-3) / 1e9 if t["t_mean_ms"] > 0 else 0.0
