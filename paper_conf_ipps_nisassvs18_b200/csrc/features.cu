@@ -113,9 +113,14 @@ k_rows(const IT *__restrict__ rp, int64_t n_rows, int64_t nnz, int64_t kh,
         over += len > kh ? (unsigned long long)(len - kh) : 0ull;
         if (len > 0) atomicOr(&rs_bits[a >> 5], 1u << (a & 31));
         if (use_hist) {
-            int64_t bin = len < hist_bins - 1 ? len : hist_bins - 1;
-            if (bin < sh_bins) atomicAdd(&s_hist[bin], 1u);
-            else atomicAdd(&hist[bin], 1ull);
+            // rows of a warp mostly share a length bin: one shared atomic per distinct bin
+            const int64_t bin = len < hist_bins - 1 ? len : hist_bins - 1;
+            const unsigned active = __activemask();
+            const unsigned same = __match_any_sync(active, (unsigned long long)bin);
+            if ((threadIdx.x & 31) == __ffs(same) - 1) {
+                if (bin < sh_bins) atomicAdd(&s_hist[bin], (unsigned)__popc(same));
+                else atomicAdd(&hist[bin], (unsigned long long)__popc(same));
+            }
         }
     }
     if (bad) atomicOr(&out->bad, bad);
@@ -130,9 +135,11 @@ k_rows(const IT *__restrict__ rp, int64_t n_rows, int64_t nnz, int64_t kh,
 }
 
 // F2: element pass -- column validity/order and the block-start bitmap.  A warp
-// handles kWordsPerIter consecutive 32-position words per iteration (all loads
-// issued before any use: the pass is a pure stream over col_idx).
-constexpr int kWordsPerIter = 8;
+// handles a chunk of 512 positions (16 words) per iteration: lane l loads its 16
+// consecutive elements with four 16-byte loads, derives 16 flag bits, and lane pairs
+// merge their half-words into the chunk's flag words.
+constexpr int kLaneElems = 16;
+constexpr int kChunkWords = kLaneElems;      // 32 lanes x 16 elements = 16 words
 
 __global__ void __launch_bounds__(kThreads)
 k_flags(const int *__restrict__ col, int64_t nnz, int64_t n_cols, int64_t n_words,
@@ -142,32 +149,38 @@ k_flags(const int *__restrict__ col, int64_t nnz, int64_t n_cols, int64_t n_word
     const int64_t n_warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const uint64_t pol = policy_evict_first();
     unsigned bad = 0;
-    for (int64_t wb = warp * kWordsPerIter; wb < n_words; wb += n_warps * kWordsPerIter) {
-        int c[kWordsPerIter];
-        unsigned rs[kWordsPerIter];
+    for (int64_t wb = warp * kChunkWords; wb < n_words; wb += n_warps * kChunkWords) {
+        const int64_t k0 = wb * 32 + (int64_t)lane * kLaneElems;      // this lane's first position
+        int c[kLaneElems];
+        if (k0 + kLaneElems <= nnz && ((uintptr_t)(col + k0) & 15) == 0) {
 #pragma unroll
-        for (int u = 0; u < kWordsPerIter; ++u) {
-            const int64_t k = (wb + u) * 32 + lane;
-            c[u] = k < nnz ? ld_hint(col + k, pol) : 0;
-            rs[u] = wb + u < n_words ? rs_bits[wb + u] : 0u;
+            for (int q = 0; q < kLaneElems / 4; ++q) {
+                const int4 v = ld_hint(reinterpret_cast<const int4 *>(col + k0) + q, pol);
+                c[4 * q] = v.x; c[4 * q + 1] = v.y; c[4 * q + 2] = v.z; c[4 * q + 3] = v.w;
+            }
+        } else {
+#pragma unroll
+            for (int e = 0; e < kLaneElems; ++e) c[e] = k0 + e < nnz ? col[k0 + e] : 0;
         }
-        const int64_t k0 = wb * 32;
-        int first_prev = (lane == 0 && k0 > 0 && k0 < nnz) ? col[k0 - 1] : 0;
+        const unsigned rw = (wb + (lane >> 1) < n_words) ? rs_bits[wb + (lane >> 1)] : 0u;
+        const unsigned rs16 = (rw >> ((lane & 1) * 16)) & 0xFFFFu;
+        int prev = __shfl_up_sync(0xffffffffu, c[kLaneElems - 1], 1);
+        if (lane == 0) prev = (k0 > 0 && k0 < nnz) ? col[k0 - 1] : 0;
+        unsigned f16 = 0;
 #pragma unroll
-        for (int u = 0; u < kWordsPerIter; ++u) {
-            const int64_t k = (wb + u) * 32 + lane;
+        for (int e = 0; e < kLaneElems; ++e) {
+            const int64_t k = k0 + e;
             const bool valid = k < nnz;
-            int prev = __shfl_up_sync(0xffffffffu, c[u], 1);
-            int last_prev_word = __shfl_sync(0xffffffffu, u > 0 ? c[u > 0 ? u - 1 : 0] : 0, 31);
-            if (lane == 0) prev = u == 0 ? first_prev : last_prev_word;
-            const bool rowstart = (rs[u] >> lane) & 1u;
-            const bool flag = valid && (rowstart || k == 0 || (int64_t)c[u] != (int64_t)prev + 1);
-            if (valid && (c[u] < 0 || (int64_t)c[u] >= n_cols)) bad |= BAD_COL_RANGE;
-            if (valid && k > 0 && !rowstart && c[u] <= prev) bad |= BAD_COL_ORDER;
+            const int pv = e == 0 ? prev : c[e - 1];
+            const bool rowstart = (rs16 >> e) & 1u;
+            const bool flag = valid && (rowstart || k == 0 || (int64_t)c[e] != (int64_t)pv + 1);
+            if (valid && (c[e] < 0 || (int64_t)c[e] >= n_cols)) bad |= BAD_COL_RANGE;
+            if (valid && k > 0 && !rowstart && c[e] <= pv) bad |= BAD_COL_ORDER;
             if (valid && k == 0 && !rowstart) bad |= BAD_ROWPTR_ORDER;
-            const unsigned fw = __ballot_sync(0xffffffffu, flag);
-            if (lane == 0 && wb + u < n_words) flag_bits[wb + u] = fw;
+            f16 |= (unsigned)flag << e;
         }
+        const unsigned hi = __shfl_down_sync(0xffffffffu, f16, 1);
+        if (!(lane & 1) && wb + (lane >> 1) < n_words) flag_bits[wb + (lane >> 1)] = f16 | (hi << 16);
     }
     bad = __reduce_or_sync(0xffffffffu, bad);
     if (lane == 0 && bad) atomicOr(&out->bad, (unsigned long long)bad);
@@ -238,55 +251,71 @@ k_scan_totals(unsigned long long *totals, int64_t n) {
     }
 }
 
-// F4: block sizes = gaps between consecutive block starts; kWordsPerIter words per
-// warp iteration (loaded up front), next start usually inside the batch, otherwise
-// a warp-cooperative forward scan (long contiguous blocks).
+// F4: block sizes = gaps between consecutive block starts.  A warp takes 256 words
+// (8192 positions) per iteration, lane l the 8 words [8l, 8l+8) loaded as two 16-byte
+// vectors; a lane walks its flags in order (gap to the previous flag = one block), the
+// block left open at the lane end closes at the first flag of a later lane (suffix
+// minimum over lanes) or, past the chunk, at the next flagged word (forward scan).
+constexpr int kLaneWords = 8;
+
 __global__ void __launch_bounds__(kThreads)
 k_block_sizes(const unsigned *__restrict__ flag_bits, int64_t n_words, int64_t nnz, FeatureSums *out) {
     const int lane = threadIdx.x & 31;
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t n_warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    constexpr int64_t CW = 32 * kLaneWords;
     unsigned long long nb = 0, sz2 = 0, mn = ULLONG_MAX, mx = 0;
-    for (int64_t wb = warp * kWordsPerIter; wb < n_words; wb += n_warps * kWordsPerIter) {
-        unsigned fw[kWordsPerIter + 1];
+    auto take = [&](unsigned long long sz) {
+        nb += 1;
+        sz2 += sz * sz;
+        mn = sz < mn ? sz : mn;
+        mx = sz > mx ? sz : mx;
+    };
+    for (int64_t wb = warp * CW; wb < n_words; wb += n_warps * CW) {
+        const int64_t w0 = wb + (int64_t)lane * kLaneWords;
+        unsigned fw[kLaneWords];
+        // flag_bits is padded to a multiple of CW words (zeros): vector loads stay inside
+        const uint4 a = *reinterpret_cast<const uint4 *>(flag_bits + w0);
+        const uint4 b = *reinterpret_cast<const uint4 *>(flag_bits + w0 + 4);
+        fw[0] = a.x; fw[1] = a.y; fw[2] = a.z; fw[3] = a.w; fw[4] = b.x; fw[5] = b.y; fw[6] = b.z; fw[7] = b.w;
+        int64_t first = -1, last = -1;
 #pragma unroll
-        for (int u = 0; u <= kWordsPerIter; ++u) fw[u] = wb + u < n_words ? flag_bits[wb + u] : 0u;
-        // next block start at or after the batch end (only needed if the tail words are flag-free)
-        unsigned any = 0;
+        for (int q = 0; q < kLaneWords; ++q) {
+            unsigned w = fw[q];
+            while (w) {
+                const int64_t p = (w0 + q) * 32 + (__ffs(w) - 1);
+                w &= w - 1;
+                if (last >= 0) take((unsigned long long)(p - last));
+                else first = p;
+                last = p;
+            }
+        }
+        // first flag strictly after this lane: suffix minimum of `first` over later lanes
+        int64_t nxt = first >= 0 ? first : INT64_MAX;
 #pragma unroll
-        for (int u = 0; u < kWordsPerIter; ++u) any |= fw[u];
-        if (!any) continue;                       // warp-uniform: no block starts in the batch
-        int64_t next_batch = nnz;
-        if (fw[kWordsPerIter]) {
-            next_batch = (wb + kWordsPerIter) * 32 + (__ffs(fw[kWordsPerIter]) - 1);
-        } else {
-            for (int64_t base = wb + kWordsPerIter + 1; base < n_words; base += 32) {
-                unsigned v = base + lane < n_words ? flag_bits[base + lane] : 0u;
-                unsigned b = __ballot_sync(0xffffffffu, v != 0u);
-                if (b) {
-                    int src = __ffs(b) - 1;
-                    unsigned fv = __shfl_sync(0xffffffffu, v, src);
-                    next_batch = (base + src) * 32 + (__ffs(fv) - 1);
+        for (int o = 1; o < 32; o <<= 1) {
+            const int64_t v = __shfl_down_sync(0xffffffffu, nxt, o);
+            if (lane + o < 32 && v < nxt) nxt = v;
+        }
+        int64_t after = __shfl_down_sync(0xffffffffu, nxt, 1);
+        if (lane == 31) after = INT64_MAX;
+        // past the chunk: the next flagged word (warp-cooperative forward scan, rare)
+        const bool need = __any_sync(0xffffffffu, last >= 0 && after == INT64_MAX);
+        if (need) {
+            int64_t beyond = nnz;
+            for (int64_t base = wb + CW; base < n_words; base += 32) {
+                const unsigned v = base + lane < n_words ? flag_bits[base + lane] : 0u;
+                const unsigned bm = __ballot_sync(0xffffffffu, v != 0u);
+                if (bm) {
+                    const int src = __ffs(bm) - 1;
+                    const unsigned fv = __shfl_sync(0xffffffffu, v, src);
+                    beyond = (base + src) * 32 + (__ffs(fv) - 1);
                     break;
                 }
             }
+            if (after == INT64_MAX) after = beyond;
         }
-        int64_t next_after = next_batch;          // next start after word u, scanning backwards
-#pragma unroll
-        for (int u = kWordsPerIter - 1; u >= 0; --u) {
-            const unsigned f = fw[u];
-            if ((f >> lane) & 1u) {
-                const unsigned above = lane == 31 ? 0u : (f & ~((2u << lane) - 1u));
-                const int64_t k = (wb + u) * 32 + lane;
-                const int64_t nxt = above ? (wb + u) * 32 + (__ffs(above) - 1) : next_after;
-                const unsigned long long sz = (unsigned long long)(nxt - k);
-                nb += 1;
-                sz2 += sz * sz;
-                mn = sz < mn ? sz : mn;
-                mx = sz > mx ? sz : mx;
-            }
-            if (f) next_after = (wb + u) * 32 + (__ffs(f) - 1);
-        }
+        if (last >= 0) take((unsigned long long)(after - last));
     }
     unsigned long long sums[2] = {nb, sz2};
     unsigned long long *g[2] = {&out->nb_tot, &out->sum_bs2};
@@ -347,7 +376,8 @@ spmv_status feature_pass_t(spmv_ctx *ctx, const spmv_csr *A, cudaStream_t s, int
     Scratch sums(ctx, s), rs(ctx, s), flags(ctx, s), local(ctx, s), totals(ctx, s), hist(ctx, s);
     SPMV_TRY(sums.alloc(sizeof(FeatureSums)));
     SPMV_TRY(rs.alloc(n_words * 4));
-    SPMV_TRY(flags.alloc(n_words * 4));
+    const int64_t n_words_pad = ceil_div<int64_t>(n_words, 256) * 256 + 256;   // F4 reads whole 256-word chunks
+    SPMV_TRY(flags.alloc(n_words_pad * 4));
     if (level) {
         SPMV_TRY(local.alloc(n_words * 4));
         SPMV_TRY(totals.alloc(n_chunks * 8));
@@ -358,6 +388,7 @@ spmv_status feature_pass_t(spmv_ctx *ctx, const spmv_csr *A, cudaStream_t s, int
     init.len_min = init.nb_min = init.bs_min = ULLONG_MAX;
     SPMV_CUDA_TRY(cudaMemcpyAsync(sums.p, &init, sizeof(init), cudaMemcpyHostToDevice, s));
     SPMV_CUDA_TRY(cudaMemsetAsync(rs.p, 0, n_words * 4, s));
+    SPMV_CUDA_TRY(cudaMemsetAsync(flags.p, 0, n_words_pad * 4, s));
     FeatureSums *d = sums.as<FeatureSums>();
 
     if (n >= 0) {
@@ -367,7 +398,7 @@ spmv_status feature_pass_t(spmv_ctx *ctx, const spmv_csr *A, cudaStream_t s, int
         SPMV_LAUNCH_CHECK();
     }
     if (n_words > 0) {
-        k_flags<<<grid_for(ctx, n_words * 32), kThreads, 0, s>>>(A->col_idx, nnz, A->n_cols, n_words,
+        k_flags<<<grid_for(ctx, ceil_div<int64_t>(n_words, kChunkWords) * 32), kThreads, 0, s>>>(A->col_idx, nnz, A->n_cols, n_words,
                                                                 rs.as<unsigned>(), flags.as<unsigned>(), d);
         SPMV_LAUNCH_CHECK();
     }
@@ -377,7 +408,7 @@ spmv_status feature_pass_t(spmv_ctx *ctx, const spmv_csr *A, cudaStream_t s, int
         SPMV_LAUNCH_CHECK();
         k_scan_totals<<<1, kThreads, 0, s>>>(totals.as<unsigned long long>(), n_chunks);
         SPMV_LAUNCH_CHECK();
-        k_block_sizes<<<grid_for(ctx, n_words * 32), kThreads, 0, s>>>(flags.as<unsigned>(), n_words, nnz, d);
+        k_block_sizes<<<grid_for(ctx, ceil_div<int64_t>(n_words, 32 * kLaneWords) * 32), kThreads, 0, s>>>(flags.as<unsigned>(), n_words, nnz, d);
         SPMV_LAUNCH_CHECK();
     }
     if (level && n > 0) {

@@ -13,6 +13,7 @@
 // in carry order (one thread per run of equal rows).
 #include <algorithm>
 #include <climits>
+#include <cstdlib>
 
 #include "internal.h"
 #include "kernels.h"
@@ -25,6 +26,7 @@ constexpr int kT = kRunThreads;
 constexpr int kIPT = kItemsPerThread;
 constexpr int kWIPT = kWarpItemsPerLane;
 constexpr int kMinBlocks = 4;   // 4 CTAs x 256 threads per SM: <= 64 registers
+constexpr int kMergeTilesPerWarp = 31;   // consecutive merge tiles per warp (coords: one load)
 constexpr int kFold = 256;   // sequential steps per accumulator before folding (A13)
 
 // ------------------------------------------------------------------ helpers
@@ -50,12 +52,13 @@ __global__ void k_scale(V *y, int64_t n, double beta) {
 
 // ------------------------------------------------------------------ CSR-vector (K3/G8)
 // "assign a WARP to process a row".  A W-lane group per row (A5).
-// One warp iteration covers R = 32 consecutive rows (U = W rows per group): their row
+// One warp iteration covers R = 32 consecutive rows (U rows per group): their row
 // pointers come from one coalesced load (+ shuffles) issued one iteration ahead
 // (software pipelined), and every group issues the first W elements of each of its U
 // rows before any x gather, so a warp keeps U independent loads per lane in flight
-// even when rows are as short as the 5-point stencil's.  Rows longer than W continue
-// in a four-accumulator loop folded every kFold steps (A13).
+// even when rows are as short as the 5-point stencil's.  Rows longer than W finish
+// with the whole warp on one row at a time (8 loads per lane in flight, accumulators
+// folded every kFold steps, A13) -- the paper's warp-per-row kernel for long rows.
 template <int W> struct VecCfg { static constexpr int U = W <= 8 ? 32 / (32 / W) : (W == 16 ? 4 : 2); };
 
 template <typename V, typename IT, int W, bool B0>
@@ -105,41 +108,6 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
         double s[U];
 #pragma unroll
         for (int u = 0; u < U; ++u) s[u] = c0[u] >= 0 ? (double)v0[u] * (double)ld_x(x + c0[u], px) : 0.0;
-        // longer rows: the rest with four accumulators (warp-uniform skip when none)
-        bool more = false;
-#pragma unroll
-        for (int u = 0; u < U; ++u) more |= (int64_t)a[u] + W < (int64_t)b[u];
-        if (__any_sync(0xffffffffu, more)) {
-#pragma unroll 1
-            for (int u = 0; u < U; ++u) {
-                const int i = u * G + g;
-                const IT au = __shfl_sync(0xffffffffu, rp_lo, i);
-                const IT nx = __shfl_sync(0xffffffffu, rp_lo, (i + 1) & 31);
-                const int64_t bu = base + i < n ? (int64_t)(i + 1 < R ? nx : rp_hi) : 0;
-                int64_t k = (int64_t)au + sub + W;
-                double tot = 0.0, a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;
-                int it = 0;
-                for (; k + 3 * W < bu; k += 4 * W) {
-                    int d0 = ld_hint(col + k, pa), d1 = ld_hint(col + k + W, pa);
-                    int d2 = ld_hint(col + k + 2 * W, pa), d3 = ld_hint(col + k + 3 * W, pa);
-                    V w0 = ld_hint(val + k, pa), w1 = ld_hint(val + k + W, pa);
-                    V w2 = ld_hint(val + k + 2 * W, pa), w3 = ld_hint(val + k + 3 * W, pa);
-                    a0 += (double)w0 * (double)ld_x(x + d0, px);
-                    a1 += (double)w1 * (double)ld_x(x + d1, px);
-                    a2 += (double)w2 * (double)ld_x(x + d2, px);
-                    a3 += (double)w3 * (double)ld_x(x + d3, px);
-                    if (++it == kFold) {                 // blocked summation (A13)
-                        tot += (a0 + a1) + (a2 + a3);
-                        a0 = a1 = a2 = a3 = 0.0;
-                        it = 0;
-                    }
-                }
-                for (; k < bu; k += W) a0 += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
-                const double extra = tot + ((a0 + a1) + (a2 + a3));
-#pragma unroll
-                for (int uu = 0; uu < U; ++uu) s[uu] += (uu == u) ? extra : 0.0;
-            }
-        }
 #pragma unroll
         for (int u = 0; u < U; ++u) {
 #pragma unroll
@@ -149,6 +117,44 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
         double mine = 0.0;
 #pragma unroll
         for (int u = 0; u < U; ++u) mine = (sub == u) ? s[u] : mine;
+        // rows longer than W: the remainder is processed by the WHOLE warp, one row at a
+        // time (the paper's warp-per-row vector kernel), 8 loads per lane in
+        // flight, accumulators folded every kFold steps (A13); lane i holds row i's range
+        {
+            const IT my_a = rp_lo;
+            const IT my_b = __shfl_sync(0xffffffffu, rp_lo, (lane + 1) & 31);
+            const IT my_e = lane + 1 < R ? my_b : rp_hi;
+            unsigned more = __ballot_sync(0xffffffffu, lane < R && base + lane < n && (int64_t)my_e - (int64_t)my_a > W);
+            while (more) {
+                const int i = __ffs(more) - 1;
+                more &= more - 1;
+                const int64_t ra = (int64_t)__shfl_sync(0xffffffffu, my_a, i) + W;
+                const int64_t rb = (int64_t)__shfl_sync(0xffffffffu, my_e, i);
+                double tot = 0.0, acc[8];
+#pragma unroll
+                for (int q = 0; q < 8; ++q) acc[q] = 0.0;
+                int it = 0;
+                int64_t k = ra + lane;
+                for (; k + 7 * 32 < rb; k += 8 * 32) {
+                    int d[8];
+                    V w[8];
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(x + d[q], px);
+                    if (++it == kFold) {                 // blocked summation (A13)
+#pragma unroll
+                        for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
+                        it = 0;
+                    }
+                }
+                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
+                double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
+                part = warp_sum(tot + part);
+                const int writer = (i % G) * W + i / G;    // lane holding row i's group sum
+                if (lane == writer) mine += part;
+            }
+        }
         if (sub < U) {
             const int64_t r = base + sub * G + g;
             if (r < n) {
@@ -184,45 +190,89 @@ k_csr_scalar(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
 
 // ------------------------------------------------------------------ ELL (K4/G9)
 // column-major, "each row is processed by a single thread".
-// Slots are consumed kEllBatch at a time with predicated loads (all in flight before
-// the first x gather); y is loaded before the slots.  Padding carries col = -1 (A3).
-constexpr int kEllBatch = 8;
+// Slots are consumed BATCH at a time with predicated loads (all in flight before the
+// first x gather); y is loaded before the slots.  RPT = 2: a thread owns two adjacent
+// rows and reads each slot pair with one 8-byte (col) and one 16-/8-byte (val) load.
+// Padding carries col = -1 (A3).
+template <typename V, int RPT> struct EllVec;
+template <typename V> struct EllVec<V, 1> {
+    using CT = int;
+    using VT = V;
+};
+template <> struct EllVec<double, 2> {
+    using CT = int2;
+    using VT = double2;
+};
+template <> struct EllVec<float, 2> {
+    using CT = int2;
+    using VT = float2;
+};
+__device__ __forceinline__ int lane_of(const int &c, int) { return c; }
+__device__ __forceinline__ int lane_of(const int2 &c, int r) { return r ? c.y : c.x; }
+template <typename V> __device__ __forceinline__ V lane_of(const V &v, int) { return v; }
+__device__ __forceinline__ double lane_of(const double2 &v, int r) { return r ? v.y : v.x; }
+__device__ __forceinline__ float lane_of(const float2 &v, int r) { return r ? v.y : v.x; }
 
-template <typename V, bool B0>
+template <typename V, bool B0, int RPT, int BATCH>
 __global__ void __launch_bounds__(kT)
 k_ell(const int *__restrict__ ecol, const V *__restrict__ eval, int64_t K, int64_t ld,
       const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta) {
+    using CT = typename EllVec<V, RPT>::CT;
+    using VT = typename EllVec<V, RPT>::VT;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
-    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
-        const double yv = B0 ? 0.0 : (double)y[r];
-        double tot = 0.0, part = 0.0;
+    const int64_t nt = ceil_div<int64_t>(n, RPT);
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nt; t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r0 = t * RPT;
+        double yv[RPT], tot[RPT], part[RPT];
+#pragma unroll
+        for (int q = 0; q < RPT; ++q) {
+            yv[q] = (!B0 && r0 + q < n) ? (double)y[r0 + q] : 0.0;
+            tot[q] = 0.0;
+            part[q] = 0.0;
+        }
         int nb = 0;
-        for (int64_t j0 = 0; j0 < K; j0 += kEllBatch) {
-            int c[kEllBatch];
-            V v[kEllBatch];
+        for (int64_t j0 = 0; j0 < K; j0 += BATCH) {
+            CT c[BATCH];
+            VT v[BATCH];
 #pragma unroll
-            for (int u = 0; u < kEllBatch; ++u) {
+            for (int u = 0; u < BATCH; ++u) {
                 const bool in = j0 + u < K;
-                c[u] = in ? ld_hint(ecol + (j0 + u) * ld + r, pa) : -1;
-                v[u] = in ? ld_hint(eval + (j0 + u) * ld + r, pa) : (V)0;
+                if (in) {
+                    c[u] = ld_hint(reinterpret_cast<const CT *>(ecol + (j0 + u) * ld + r0), pa);
+                    v[u] = ld_hint(reinterpret_cast<const VT *>(eval + (j0 + u) * ld + r0), pa);
+                } else {
+                    c[u] = CT{};
+                    v[u] = VT{};
+                }
             }
-            double a0 = 0.0, a1 = 0.0;
 #pragma unroll
-            for (int u = 0; u < kEllBatch; u += 2) {
-                if (c[u] >= 0) a0 += (double)v[u] * (double)ld_x(x + c[u], px);
-                if (c[u + 1] >= 0) a1 += (double)v[u + 1] * (double)ld_x(x + c[u + 1], px);
+            for (int q = 0; q < RPT; ++q) {
+                double a0 = 0.0, a1 = 0.0;
+#pragma unroll
+                for (int u = 0; u < BATCH; u += 2) {
+                    const int cu = lane_of(c[u], q);
+                    if (j0 + u < K && cu >= 0) a0 += (double)lane_of(v[u], q) * (double)ld_x(x + cu, px);
+                    if (u + 1 < BATCH) {
+                        const int cw = lane_of(c[u + 1], q);
+                        if (j0 + u + 1 < K && cw >= 0) a1 += (double)lane_of(v[u + 1], q) * (double)ld_x(x + cw, px);
+                    }
+                }
+                part[q] += a0 + a1;
             }
-            part += a0 + a1;
             if (++nb == kFold) {                          // blocked summation (A13)
-                tot += part;
-                part = 0.0;
+#pragma unroll
+                for (int q = 0; q < RPT; ++q) { tot[q] += part[q]; part[q] = 0.0; }
                 nb = 0;
             }
         }
-        tot += part;
-        double o = alpha * tot;
-        if (!B0) o = fma(beta, yv, o);
-        y[r] = (V)o;
+#pragma unroll
+        for (int q = 0; q < RPT; ++q) {
+            if (r0 + q < n) {
+                double o = alpha * (tot[q] + part[q]);
+                if (!B0) o = fma(beta, yv[q], o);
+                y[r0 + q] = (V)o;
+            }
+        }
     }
 }
 
@@ -465,8 +515,8 @@ __device__ __forceinline__ void shift_load_int8(const int *p, int (&v)[8], uint6
     for (int s = 0; s < 8; ++s) v[s] = m == 0 ? w[s] : m == 1 ? w[s + 1] : m == 2 ? w[s + 2] : w[s + 3];
 }
 
-template <typename V, typename IT, bool B0>
-__global__ void __launch_bounds__(kT, kMinBlocks)
+template <typename V, typename IT, bool B0, int MB>
+__global__ void __launch_bounds__(kT, MB)
 k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
         const int64_t *__restrict__ crow, const int64_t *__restrict__ cnz, int64_t n_tiles, int64_t n_rows,
         const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
@@ -479,15 +529,24 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
     __shared__ unsigned s_flag_all[kT / 32][TI / 32];
     __shared__ unsigned s_mark_all[kT / 32][TI / 32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    if (t >= n_tiles) return;
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t tbase = gw * kMergeTilesPerWarp;
+    if (tbase >= n_tiles) return;
     double *s_sum = s_sum_all[wid];
     int *s_end = s_end_all[wid];
     unsigned short *s_rowat = s_rowat_all[wid];
     unsigned *s_flag = s_flag_all[wid];
     unsigned *s_mark = s_mark_all[wid];
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
-    const int64_t r0 = __ldg(crow + t), k0 = __ldg(cnz + t), r1 = __ldg(crow + t + 1), k1 = __ldg(cnz + t + 1);
+    // the warp owns kMergeTilesPerWarp consecutive tiles: all their coordinates in one
+    // coalesced load (lane j holds the coordinate at the start of tile tbase + j)
+    const int64_t cidx = tbase + lane <= n_tiles ? tbase + lane : n_tiles;
+    const int64_t c_row = __ldg(crow + cidx), c_nz = __ldg(cnz + cidx);
+    const int ntw = (int)(n_tiles - tbase < kMergeTilesPerWarp ? n_tiles - tbase : kMergeTilesPerWarp);
+    for (int tj = 0; tj < ntw; ++tj) {
+    const int64_t t = tbase + tj;
+    const int64_t r0 = __shfl_sync(0xffffffffu, c_row, tj), k0 = __shfl_sync(0xffffffffu, c_nz, tj);
+    const int64_t r1 = __shfl_sync(0xffffffffu, c_row, tj + 1), k1 = __shfl_sync(0xffffffffu, c_nz, tj + 1);
     const int nrows = (int)(r1 - r0), nnzt = (int)(k1 - k0);
     const int j0 = lane * 8;
     const int nv = max(0, min(8, nnzt - j0));
@@ -572,6 +631,8 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
         double o = marked ? alpha * s_sum[i] : 0.0;
         if (!B0) o = fma(beta, (double)y[r0 + i], o);
         y[r0 + i] = (V)o;
+    }
+    __syncwarp();                                         // the shared slice is reused by the next tile
     }
 }
 
@@ -775,6 +836,24 @@ spmv_status launch_fixup(spmv_handle *h, V *y, double alpha, cudaStream_t s) {
     return SPMV_OK;
 }
 
+// ELL variant: rows per thread x slot batch (SPMV_ELL_VARIANT = "RB", e.g. "18", "24")
+template <typename V, bool B0>
+spmv_status launch_ell(spmv_handle *h, const V *x, V *y, double alpha, double beta, cudaStream_t s) {
+    const int64_t n = h->n_rows;
+    if (n == 0) return SPMV_OK;
+    static const int var = [] { const char *e = getenv("SPMV_ELL_VARIANT"); return e ? atoi(e) : 18; }();
+    const int *c = (const int *)h->arr[SPMV_ARR_ELL_COL].p;
+    const V *v = (const V *)h->arr[SPMV_ARR_ELL_VAL].p;
+    switch (var) {
+    case 14: k_ell<V, B0, 1, 4><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
+    case 24: k_ell<V, B0, 2, 4><<<grid_stride_blocks(h->ctx, (n + 1) / 2, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
+    case 28: k_ell<V, B0, 2, 8><<<grid_stride_blocks(h->ctx, (n + 1) / 2, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
+    default: k_ell<V, B0, 1, 8><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
+    }
+    SPMV_LAUNCH_CHECK();
+    return SPMV_OK;
+}
+
 template <typename V, typename IT, bool B0>
 spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col, const V *val, const V *x, V *y,
                               int64_t n, int w, double alpha, double beta, cudaStream_t s) {
@@ -814,17 +893,10 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
         return SPMV_OK;
     case SPMV_ELL:
         if (n == 0) return SPMV_OK;
-        k_ell<V, B0><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(
-            (const int *)h->arr[SPMV_ARR_ELL_COL].p, (const V *)h->arr[SPMV_ARR_ELL_VAL].p, h->ell_K, h->ell_ld,
-            x, y, n, alpha, beta);
-        SPMV_LAUNCH_CHECK();
-        return SPMV_OK;
+        return launch_ell<V, B0>(h, x, y, alpha, beta, s);
     case SPMV_HYB: {
         if (n == 0) return SPMV_OK;
-        k_ell<V, B0><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(
-            (const int *)h->arr[SPMV_ARR_ELL_COL].p, (const V *)h->arr[SPMV_ARR_ELL_VAL].p, h->ell_K, h->ell_ld,
-            x, y, n, alpha, beta);
-        SPMV_LAUNCH_CHECK();
+        SPMV_TRY((launch_ell<V, B0>(h, x, y, alpha, beta, s)));
         if (h->hyb_coo_nnz == 0) return SPMV_OK;
         k_coo<V, true, B0><<<(unsigned)ceil_div<int64_t>(h->n_carry, kT / 32), kT, 0, s>>>(
             (const int *)h->arr[SPMV_ARR_COO_ROW].p, (const int *)h->arr[SPMV_ARR_HYB_COO_COL].p,
@@ -840,9 +912,16 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
         return launch_fixup<V>(h, y, alpha, s);
     case SPMV_MERGE:
         if (h->merge_tiles == 0) return SPMV_OK;
-        k_merge<V, IT, B0><<<(unsigned)ceil_div<int64_t>(h->merge_tiles, kT / 32), kT, 0, s>>>(
-            rp, col, val, (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_ROW].p,
-            (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_NZ].p, h->merge_tiles, n, x, y, alpha, beta, crow, cval);
+    {
+        static const int mb = [] { const char *e = getenv("SPMV_MERGE_MB"); return e ? atoi(e) : 4; }();
+        const unsigned g = (unsigned)ceil_div<int64_t>(h->merge_tiles, (kT / 32) * kMergeTilesPerWarp);
+        const int64_t *cr = (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_ROW].p;
+        const int64_t *cz = (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_NZ].p;
+        if (mb == 3)
+            k_merge<V, IT, B0, 3><<<g, kT, 0, s>>>(rp, col, val, cr, cz, h->merge_tiles, n, x, y, alpha, beta, crow, cval);
+        else
+            k_merge<V, IT, B0, 4><<<g, kT, 0, s>>>(rp, col, val, cr, cz, h->merge_tiles, n, x, y, alpha, beta, crow, cval);
+    }
         SPMV_LAUNCH_CHECK();
         return launch_fixup<V>(h, y, alpha, s);
     case SPMV_CSR5: {
