@@ -99,6 +99,14 @@ __device__ __forceinline__ double2 ld_hint(const double2 *p, uint64_t pol) {
                  : "=d"(v.x), "=d"(v.y) : "l"(p), "l"(pol));
     return v;
 }
+// four doubles (two 16-byte loads) -- ELL's 4-rows-per-thread slot pairs
+struct double4a { double2 lo, hi; };
+__device__ __forceinline__ double4a ld_hint(const double4a *p, uint64_t pol) {
+    double4a r;
+    r.lo = ld_hint(reinterpret_cast<const double2 *>(p), pol);
+    r.hi = ld_hint(reinterpret_cast<const double2 *>(p) + 1, pol);
+    return r;
+}
 // x gathers: read-only path, keep in L1 (neighbouring gathers hit), L2 evict-last
 __device__ __forceinline__ float ld_x(const float *p, uint64_t pol) {
     float v;

@@ -365,8 +365,8 @@ spmv_status convert_t(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, const s
     case SPMV_MERGE: {
         SPMV_TRY(copy_colval(false));   // padded copies: the kernel's shifted vector loads need the slack
         int64_t T = o->merge_items > 0 ? o->merge_items : kMergeItems;
-        if (T != kMergeItems) {
-            set_error("merge_items other than the compiled tile size is not supported");
+        if (T != 128 && T != 256) {
+            set_error("merge_items must be 128 or 256 (32 lanes x 4 or 8 items)");
             return SPMV_ERR_UNSUPPORTED;
         }
         int64_t tiles = ceil_div<int64_t>(n + nnz, T);

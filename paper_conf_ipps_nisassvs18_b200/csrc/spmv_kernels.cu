@@ -26,7 +26,6 @@ constexpr int kT = kRunThreads;
 constexpr int kIPT = kItemsPerThread;
 constexpr int kWIPT = kWarpItemsPerLane;
 constexpr int kMinBlocks = 4;   // 4 CTAs x 256 threads per SM: <= 64 registers
-constexpr int kMergeTilesPerWarp = 31;   // consecutive merge tiles per warp (coords: one load)
 constexpr int kFold = 256;   // sequential steps per accumulator before folding (A13)
 
 // ------------------------------------------------------------------ helpers
@@ -207,8 +206,20 @@ template <> struct EllVec<float, 2> {
     using CT = int2;
     using VT = float2;
 };
+template <> struct EllVec<double, 4> {
+    using CT = int4;
+    using VT = double4a;
+};
+template <> struct EllVec<float, 4> {
+    using CT = int4;
+    using VT = float4;
+};
 __device__ __forceinline__ int lane_of(const int &c, int) { return c; }
 __device__ __forceinline__ int lane_of(const int2 &c, int r) { return r ? c.y : c.x; }
+__device__ __forceinline__ int lane_of(const int4 &c, int r) { return r == 0 ? c.x : r == 1 ? c.y : r == 2 ? c.z : c.w; }
+__device__ __forceinline__ double lane_of(const double4a &v, int r) { return r == 0 ? v.lo.x : r == 1 ? v.lo.y : r == 2 ? v.hi.x : v.hi.y; }
+__device__ __forceinline__ float lane_of(const float4 &v, int r) { return r == 0 ? v.x : r == 1 ? v.y : r == 2 ? v.z : v.w; }
+
 template <typename V> __device__ __forceinline__ V lane_of(const V &v, int) { return v; }
 __device__ __forceinline__ double lane_of(const double2 &v, int r) { return r ? v.y : v.x; }
 __device__ __forceinline__ float lane_of(const float2 &v, int r) { return r ? v.y : v.x; }
@@ -482,79 +493,68 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
 // in the tile is written by it (empty rows: beta*y); row r0 may have begun in an
 // earlier tile (its earlier parts arrive as carries); the part of row r1 inside the
 // tile is the tile carry.  The row window is written back coalesced.
-template <typename V> struct ShiftLoad8;
-template <> struct ShiftLoad8<double> {    // 8 doubles from p (8-byte aligned): 5 x double2, shift 0/1
-    static __device__ __forceinline__ void load(const double *p, double (&v)[8], uint64_t pol) {
+// N consecutive elements starting at an arbitrary (element-aligned) address: the
+// covering 16-byte vectors, then a shift by the address's offset inside a vector
+template <typename V, int N> struct ShiftLoad;
+template <int N> struct ShiftLoad<double, N> {          // N/2 + 1 double2, shift 0/1
+    static __device__ __forceinline__ void load(const double *p, double (&v)[N], uint64_t pol) {
         const int m = (int)(((uintptr_t)p >> 3) & 1);
         const double2 *b = reinterpret_cast<const double2 *>(p - m);
-        double w[10];
+        double w[N + 2];
 #pragma unroll
-        for (int q = 0; q < 5; ++q) { double2 t = ld_hint(b + q, pol); w[2 * q] = t.x; w[2 * q + 1] = t.y; }
+        for (int q = 0; q < N / 2 + 1; ++q) { double2 t = ld_hint(b + q, pol); w[2 * q] = t.x; w[2 * q + 1] = t.y; }
 #pragma unroll
-        for (int s = 0; s < 8; ++s) v[s] = m ? w[s + 1] : w[s];
+        for (int s = 0; s < N; ++s) v[s] = m ? w[s + 1] : w[s];
     }
 };
-template <> struct ShiftLoad8<float> {     // 8 floats: 3 x float4, shift 0..3
-    static __device__ __forceinline__ void load(const float *p, float (&v)[8], uint64_t pol) {
-        const int m = (int)(((uintptr_t)p >> 2) & 3);
-        const float4 *b = reinterpret_cast<const float4 *>(p - m);
-        float w[12];
-#pragma unroll
-        for (int q = 0; q < 3; ++q) { float4 t = ld_hint(b + q, pol); w[4*q] = t.x; w[4*q+1] = t.y; w[4*q+2] = t.z; w[4*q+3] = t.w; }
-#pragma unroll
-        for (int s = 0; s < 8; ++s) v[s] = m == 0 ? w[s] : m == 1 ? w[s + 1] : m == 2 ? w[s + 2] : w[s + 3];
-    }
-};
-__device__ __forceinline__ void shift_load_int8(const int *p, int (&v)[8], uint64_t pol) {
+template <typename T, typename T4, int N>
+__device__ __forceinline__ void shift_load4(const T *p, T (&v)[N], uint64_t pol) {   // N/4 + 1 x 16 B, shift 0..3
     const int m = (int)(((uintptr_t)p >> 2) & 3);
-    const int4 *b = reinterpret_cast<const int4 *>(p - m);
-    int w[12];
+    const T4 *b = reinterpret_cast<const T4 *>(p - m);
+    T w[N + 4];
 #pragma unroll
-    for (int q = 0; q < 3; ++q) { int4 t = ld_hint(b + q, pol); w[4*q] = t.x; w[4*q+1] = t.y; w[4*q+2] = t.z; w[4*q+3] = t.w; }
+    for (int q = 0; q < N / 4 + 1; ++q) { T4 t = ld_hint(b + q, pol); w[4*q] = t.x; w[4*q+1] = t.y; w[4*q+2] = t.z; w[4*q+3] = t.w; }
 #pragma unroll
-    for (int s = 0; s < 8; ++s) v[s] = m == 0 ? w[s] : m == 1 ? w[s + 1] : m == 2 ? w[s + 2] : w[s + 3];
+    for (int s = 0; s < N; ++s) v[s] = m == 0 ? w[s] : m == 1 ? w[s + 1] : m == 2 ? w[s + 2] : w[s + 3];
 }
+template <int N> struct ShiftLoad<float, N> {
+    static __device__ __forceinline__ void load(const float *p, float (&v)[N], uint64_t pol) { shift_load4<float, float4, N>(p, v, pol); }
+};
+template <int N> struct ShiftLoad<int, N> {
+    static __device__ __forceinline__ void load(const int *p, int (&v)[N], uint64_t pol) { shift_load4<int, int4, N>(p, v, pol); }
+};
 
-template <typename V, typename IT, bool B0, int MB>
-__global__ void __launch_bounds__(kT, MB)
+template <typename V, typename IT, bool B0, int LI>
+__global__ void __launch_bounds__(kT, LI == 4 ? 6 : kMinBlocks)
 k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
         const int64_t *__restrict__ crow, const int64_t *__restrict__ cnz, int64_t n_tiles, int64_t n_rows,
         const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
         int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
-    constexpr int TI = (int)kMergeItems;
-    static_assert(TI == 256 && kWIPT == 8, "merge tile is 32 lanes x 8");
+    constexpr int TI = 32 * LI;                           // merge-path items per warp tile
+    static_assert(LI == 4 || LI == 8, "lane chunk of 4 or 8 items");
     __shared__ double s_sum_all[kT / 32][TI];             // row sums (local row index)
     __shared__ int s_end_all[kT / 32][TI];                // local end of local row i
     __shared__ unsigned short s_rowat_all[kT / 32][TI];   // local row starting at a position
     __shared__ unsigned s_flag_all[kT / 32][TI / 32];
     __shared__ unsigned s_mark_all[kT / 32][TI / 32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t tbase = gw * kMergeTilesPerWarp;
-    if (tbase >= n_tiles) return;
+    const int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    if (t >= n_tiles) return;
     double *s_sum = s_sum_all[wid];
     int *s_end = s_end_all[wid];
     unsigned short *s_rowat = s_rowat_all[wid];
     unsigned *s_flag = s_flag_all[wid];
     unsigned *s_mark = s_mark_all[wid];
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
-    // the warp owns kMergeTilesPerWarp consecutive tiles: all their coordinates in one
-    // coalesced load (lane j holds the coordinate at the start of tile tbase + j)
-    const int64_t cidx = tbase + lane <= n_tiles ? tbase + lane : n_tiles;
-    const int64_t c_row = __ldg(crow + cidx), c_nz = __ldg(cnz + cidx);
-    const int ntw = (int)(n_tiles - tbase < kMergeTilesPerWarp ? n_tiles - tbase : kMergeTilesPerWarp);
-    for (int tj = 0; tj < ntw; ++tj) {
-    const int64_t t = tbase + tj;
-    const int64_t r0 = __shfl_sync(0xffffffffu, c_row, tj), k0 = __shfl_sync(0xffffffffu, c_nz, tj);
-    const int64_t r1 = __shfl_sync(0xffffffffu, c_row, tj + 1), k1 = __shfl_sync(0xffffffffu, c_nz, tj + 1);
+    const int64_t r0 = __ldg(crow + t), k0 = __ldg(cnz + t), r1 = __ldg(crow + t + 1), k1 = __ldg(cnz + t + 1);
     const int nrows = (int)(r1 - r0), nnzt = (int)(k1 - k0);
-    const int j0 = lane * 8;
-    const int nv = max(0, min(8, nnzt - j0));
-    int c[8];
-    V v[8];
+    const int j0 = lane * LI;
+    const int nv = max(0, min(LI, nnzt - j0));
+    int c[LI];
+    V v[LI];
     if (nv > 0) {
-        shift_load_int8(col + k0 + j0, c, pa);
-        ShiftLoad8<V>::load(val + k0 + j0, v, pa);
+        ShiftLoad<int, LI>::load(col + k0 + j0, c, pa);
+        ShiftLoad<V, LI>::load(val + k0 + j0, v, pa);
     }
     double yv[kOutQ];
 #pragma unroll
@@ -565,9 +565,9 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
     for (int i = lane; i < nrows; i += 32) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
     const bool r0_inside = (int64_t)__ldg(rp + r0) == k0;   // A7: rp[r0] <= k0 always
     if (lane < TI / 32) { s_flag[lane] = 0u; s_mark[lane] = 0u; }
-    double p[8];
+    double p[LI];
 #pragma unroll
-    for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
+    for (int s = 0; s < LI; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
     __syncwarp();
     // segment starts: local row i (1 <= i <= nrows) starts at s_end[i-1]; row 0 at 0 if r0_inside
     for (int i = lane; i <= nrows; i += 32) {
@@ -579,7 +579,7 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
         }
     }
     __syncwarp();
-    const unsigned fl = nv > 0 ? ((s_flag[j0 >> 5] >> (j0 & 31)) & 0xFFu) : 0u;
+    const unsigned fl = nv > 0 ? ((s_flag[j0 >> 5] >> (j0 & 31)) & ((1u << LI) - 1u)) : 0u;
     auto put = [&](int li, double sum) {
         s_sum[li] = sum;
         atomicOr(&s_mark[li >> 5], 1u << (li & 31));
@@ -587,7 +587,7 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
     double acc = 0.0, head = 0.0;
     int kseg = 0, cur = -1;
 #pragma unroll
-    for (int s = 0; s < 8; ++s) {
+    for (int s = 0; s < LI; ++s) {
         if ((fl >> s) & 1u) {
             if (kseg == 0) head = acc;
             else put(cur, acc);                           // closed inside the lane (cur < nrows)
@@ -631,8 +631,6 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
         double o = marked ? alpha * s_sum[i] : 0.0;
         if (!B0) o = fma(beta, (double)y[r0 + i], o);
         y[r0 + i] = (V)o;
-    }
-    __syncwarp();                                         // the shared slice is reused by the next tile
     }
 }
 
@@ -836,19 +834,27 @@ spmv_status launch_fixup(spmv_handle *h, V *y, double alpha, cudaStream_t s) {
     return SPMV_OK;
 }
 
-// ELL variant: rows per thread x slot batch (SPMV_ELL_VARIANT = "RB", e.g. "18", "24")
+// ELL rows-per-thread x slot-batch variant; SPMV_ELL_VARIANT="RB" (e.g. 18, 24, 42) overrides the
+// dtype default for tuning experiments (tools/exp.py)
 template <typename V, bool B0>
 spmv_status launch_ell(spmv_handle *h, const V *x, V *y, double alpha, double beta, cudaStream_t s) {
     const int64_t n = h->n_rows;
     if (n == 0) return SPMV_OK;
-    static const int var = [] { const char *e = getenv("SPMV_ELL_VARIANT"); return e ? atoi(e) : 18; }();
+    static const int var = [] { const char *e = getenv("SPMV_ELL_VARIANT"); return e ? atoi(e) : 0; }();
     const int *c = (const int *)h->arr[SPMV_ARR_ELL_COL].p;
     const V *v = (const V *)h->arr[SPMV_ARR_ELL_VAL].p;
     switch (var) {
     case 14: k_ell<V, B0, 1, 4><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
-    case 24: k_ell<V, B0, 2, 4><<<grid_stride_blocks(h->ctx, (n + 1) / 2, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
     case 28: k_ell<V, B0, 2, 8><<<grid_stride_blocks(h->ctx, (n + 1) / 2, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
-    default: k_ell<V, B0, 1, 8><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
+    case 42: k_ell<V, B0, 4, 2><<<grid_stride_blocks(h->ctx, (n + 3) / 4, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
+    case 44: k_ell<V, B0, 4, 4><<<grid_stride_blocks(h->ctx, (n + 3) / 4, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
+    case 18: k_ell<V, B0, 1, 8><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
+    default:   // 16-byte value loads: fp64 2 rows x 4-slot batch, fp32 4 rows x 2-slot batch (measured best)
+        if (sizeof(V) == 8)
+            k_ell<V, B0, 2, 4><<<grid_stride_blocks(h->ctx, (n + 1) / 2, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta);
+        else
+            k_ell<V, B0, 4, 2><<<grid_stride_blocks(h->ctx, (n + 3) / 4, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta);
+        break;
     }
     SPMV_LAUNCH_CHECK();
     return SPMV_OK;
@@ -913,14 +919,13 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
     case SPMV_MERGE:
         if (h->merge_tiles == 0) return SPMV_OK;
     {
-        static const int mb = [] { const char *e = getenv("SPMV_MERGE_MB"); return e ? atoi(e) : 4; }();
-        const unsigned g = (unsigned)ceil_div<int64_t>(h->merge_tiles, (kT / 32) * kMergeTilesPerWarp);
+        const unsigned g = (unsigned)ceil_div<int64_t>(h->merge_tiles, kT / 32);
         const int64_t *cr = (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_ROW].p;
         const int64_t *cz = (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_NZ].p;
-        if (mb == 3)
-            k_merge<V, IT, B0, 3><<<g, kT, 0, s>>>(rp, col, val, cr, cz, h->merge_tiles, n, x, y, alpha, beta, crow, cval);
-        else
+        if (h->merge_T == 128)
             k_merge<V, IT, B0, 4><<<g, kT, 0, s>>>(rp, col, val, cr, cz, h->merge_tiles, n, x, y, alpha, beta, crow, cval);
+        else
+            k_merge<V, IT, B0, 8><<<g, kT, 0, s>>>(rp, col, val, cr, cz, h->merge_tiles, n, x, y, alpha, beta, crow, cval);
     }
         SPMV_LAUNCH_CHECK();
         return launch_fixup<V>(h, y, alpha, s);
