@@ -231,16 +231,17 @@ def run_ours(args):
     feat_ms = fe0.elapsed_time(fe1)
 
     # ---- partition (a14) for N > 1: this rank's rows, columns remapped to gathered-x slots
+    # (DistSpMV: merge-path row splits, shard, optional compressed exchange)
     dsp = None
     if ws > 1:
-        from paper_conf_ipps_nisassvs18_b200.dist import ShardLayout, all_gather_slots
-        splits = sp.partition(dA, ws)
-        lay = ShardLayout(splits, rank)
-        local_A, S = sp.slice_remap(dA, splits, rank)
-        x_local = lay.pack_x(torch.from_numpy(x_h[lay.r0:lay.r1].copy()).cuda().to(dtype))
-        x_run = torch.zeros(S * ws, dtype=dtype, device="cuda")
+        from paper_conf_ipps_nisassvs18_b200.dist import DistSpMV
+        dsp = DistSpMV(dA, formats[0] if args.formats else "csr5", compress=args.compress)
+        lay = dsp.layout
+        local_A = dsp.shard
+        dsp.set_x(torch.from_numpy(x_h[lay.r0:lay.r1].copy()).cuda().to(dtype))
+        x_run = dsp.x_gathered
         y_init = torch.from_numpy(y_h[lay.r0:lay.r1].copy()).cuda().to(dtype)
-        dsp = (lay, all_gather_slots)
+        S = dsp.slot
     else:
         local_A = dA
         x_run = torch.from_numpy(x_h).cuda().to(dtype)
@@ -269,7 +270,7 @@ def run_ours(args):
     # configuration is tests/test_gpu_parity.py::test_full_size_lap4096): all formats
     # agree, and for the Laplacian the closed form A*1 = {0 interior, 1 edge, 2 corner}
     if ws > 1:
-        dsp[1](x_run, x_local)
+        dsp.exchange()
     probe = {}
     for f in fmts:
         yp = y_init.clone()
@@ -303,7 +304,7 @@ def run_ours(args):
 
     def step(record=None):
         if ws > 1:
-            dsp[1](x_run, x_local)                 # the step's x all-gather (NCCL)
+            dsp.exchange()                         # the step's x all-gather (NCCL)
         for f in fmts:
             if record is not None:
                 record[f][0].record(stream)
@@ -394,7 +395,9 @@ def run_ours(args):
                        "n_rows": A.n_rows, "n_cols": A.n_cols, "nnz": A.nnz, "formats": fmts,
                        "step": "one SpMV (alpha=1, beta=1) in each feasible format",
                        "l2": "no flush: every format's arrays exceed the 126 MB L2",
-                       "parallelism": f"row-partitioned x{ws}, NCCL all-gather of x" if ws > 1 else "1 GPU"},
+                       "parallelism": (f"row-partitioned x{ws}, NCCL all-gather of x"
+                                       + (" (compressed)" if args.compress else "")) if ws > 1 else "1 GPU",
+                       "exchange_bytes_per_rank": dsp.exchange_bytes() if dsp is not None else 0},
             "per_format": per_format, "best_format": best,
             "roofline": roof(dom), "roofline_best": roof(best),
             "features": {"ms": feat_ms, "gbs": (4 * A.nnz + 8 * (A.n_rows + 1)) / (feat_ms * 1e-3) / 1e9,
@@ -431,6 +434,7 @@ def main():
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--formats", default="")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--compress", action="store_true", help="N > 1: exchange only referenced columns")
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0)

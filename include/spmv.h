@@ -240,6 +240,32 @@ spmv_status spmv_slice_remap(spmv_ctx *ctx, const spmv_csr *A, const int64_t *ro
                              int nparts, int part, void *stream,
                              int32_t *row_ptr_out, int32_t *col_out, void *vals_out);
 
+/* Compressed exchange: only columns that some row of A references are
+ * exchanged.  colmap_out[j] (DEVICE, int32[n_cols]) = owner(j)*S' + (number of referenced
+ * columns of owner(j) before j) for a referenced column j, -1 for a column no row uses;
+ * S' = max over parts of referenced columns per part (host output *slot).  Square A.
+ * Identical on every rank for the same A.  Blocks on `stream` (one readback). */
+spmv_status spmv_partition_colmap(spmv_ctx *ctx, const spmv_csr *A, const int64_t *row_splits_host,
+                                  int nparts, void *stream, int32_t *colmap_out, int64_t *slot);
+
+/* Shard `part` like spmv_slice_remap, with columns mapped through `colmap` (DEVICE,
+ * from spmv_partition_colmap) instead of the dense slot layout.  Asynchronous. */
+spmv_status spmv_slice_remap_colmap(spmv_ctx *ctx, const spmv_csr *A, const int64_t *row_splits_host,
+                                    int nparts, int part, const int32_t *colmap, void *stream,
+                                    int32_t *row_ptr_out, int32_t *col_out, void *vals_out);
+
+/* Local positions of part `part`'s referenced columns, in order: idx_out[q] = j - splits[part]
+ * for the q-th referenced column j of the part (DEVICE int32 output, capacity = part rows);
+ * `slot` is S' from spmv_partition_colmap; *count (host) = number written.  Blocks on `stream`. */
+spmv_status spmv_colmap_pack_index(spmv_ctx *ctx, const int32_t *colmap, const int64_t *row_splits_host,
+                                   int nparts, int part, int64_t slot, void *stream, int32_t *idx_out,
+                                   int64_t *count);
+
+/* dst[q] = src[idx[q]] for q < n (DEVICE arrays of `dtype`): the per-step packing of a
+ * rank's x slice into its compressed slot.  Asynchronous. */
+spmv_status spmv_gather(spmv_ctx *ctx, spmv_dtype dtype, const void *src, const int32_t *idx, int64_t n,
+                        void *dst, void *stream);
+
 /* ---- diagnostics ----------------------------------------------------------- */
 const char *spmv_status_str(spmv_status s);
 const char *spmv_last_error(void);

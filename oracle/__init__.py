@@ -88,6 +88,8 @@ def lib():
             "ora_partition": (C.c_int, [_i64, _p, C.c_int, _p]),
             "ora_partition_slot": (_i64, [_p, C.c_int]),
             "ora_slice_remap": (C.c_int, [_i64, _p, _p, _p, _p, C.c_int, C.c_int, _p, _p, _p]),
+            "ora_partition_colmap": (_i64, [_i64, _p, _p, _p, C.c_int, _p]),
+            "ora_slice_remap_colmap": (C.c_int, [_i64, _p, _p, _p, _p, C.c_int, _p, _p, _p, _p]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -298,6 +300,29 @@ def slice_remap(A, splits, part):
     rc = lib().ora_slice_remap(A.n_rows, _ptr(A.row_ptr), _ptr(A.col), _ptr(A.val), _ptr(s), P,
                                int(part), _ptr(rp), _ptr(col), _ptr(val))
     assert rc == 0, rc
+    return rp, col, val
+
+
+def partition_colmap(A, splits):
+    """Compressed-exchange column map and slot size S'."""
+    A = CSR.of(A)
+    s = _c(splits, np.int64)
+    cm = _buf(A.n_rows, np.int32)
+    S = lib().ora_partition_colmap(A.n_rows, _ptr(A.row_ptr), _ptr(A.col), _ptr(s), s.size - 1, _ptr(cm))
+    assert S >= 0
+    return cm, int(S)
+
+
+def slice_remap_colmap(A, splits, part, colmap):
+    A = CSR.of(A)
+    s = _c(splits, np.int64)
+    cm = _c(colmap, np.int32)
+    r0, r1 = int(s[part]), int(s[part + 1])
+    nnz_p = int(A.row_ptr[r1] - A.row_ptr[r0])
+    rp, col, val = _buf(r1 - r0 + 1, np.int64), _buf(nnz_p, np.int32), _buf(nnz_p, np.float64)
+    rc = lib().ora_slice_remap_colmap(A.n_rows, _ptr(A.row_ptr), _ptr(A.col), _ptr(A.val), _ptr(s), int(part),
+                                      _ptr(cm), _ptr(rp), _ptr(col), _ptr(val))
+    assert rc == 0
     return rp, col, val
 
 

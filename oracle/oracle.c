@@ -537,3 +537,40 @@ int ora_slice_remap(int64_t n_rows, const int64_t *row_ptr, const int32_t *col,
     }
     return 0;
 }
+
+/* Compressed exchange: a column is exchanged only if some row references it. */
+int64_t ora_partition_colmap(int64_t n_rows, const int64_t *row_ptr, const int32_t *col,
+                             const int64_t *splits, int nparts, int32_t *colmap)
+{
+    int64_t nnz = row_ptr[n_rows];
+    unsigned char *used = (unsigned char *)calloc((size_t)(n_rows > 0 ? n_rows : 1), 1);
+    if (!used) return -1;
+    for (int64_t k = 0; k < nnz; ++k) used[col[k]] = 1;
+    int64_t S = 0;
+    for (int part = 0; part < nparts; ++part) {
+        int64_t c = 0;
+        for (int64_t j = splits[part]; j < splits[part + 1]; ++j) c += used[j];
+        if (c > S) S = c;
+    }
+    for (int part = 0; part < nparts; ++part) {
+        int64_t c = 0;
+        for (int64_t j = splits[part]; j < splits[part + 1]; ++j)
+            colmap[j] = used[j] ? (int32_t)(part * S + c++) : -1;
+    }
+    free(used);
+    return S;
+}
+
+int ora_slice_remap_colmap(int64_t n_rows, const int64_t *row_ptr, const int32_t *col,
+                           const double *val, const int64_t *splits, int part, const int32_t *colmap,
+                           int64_t *out_row_ptr, int32_t *out_col, double *out_val)
+{
+    int64_t r0 = splits[part], r1 = splits[part + 1];
+    if (r1 > n_rows) return -1;
+    for (int64_t r = r0; r <= r1; ++r) out_row_ptr[r - r0] = row_ptr[r] - row_ptr[r0];
+    for (int64_t k = row_ptr[r0]; k < row_ptr[r1]; ++k) {
+        out_col[k - row_ptr[r0]] = colmap[col[k]];
+        out_val[k - row_ptr[r0]] = val[k];
+    }
+    return 0;
+}

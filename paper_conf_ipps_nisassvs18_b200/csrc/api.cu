@@ -317,4 +317,45 @@ spmv_status spmv_slice_remap(spmv_ctx *ctx, const spmv_csr *A, const int64_t *sp
     return slice_remap_impl(ctx, A, splits, nparts, part, as_stream(stream), rp_out, col_out, val_out);
 }
 
+spmv_status spmv_partition_colmap(spmv_ctx *ctx, const spmv_csr *A, const int64_t *splits, int nparts, void *stream,
+                                  int32_t *colmap_out, int64_t *slot) {
+    if (!ctx || !splits || nparts <= 0 || !colmap_out || !slot) { set_error("bad args"); return SPMV_ERR_INVALID_ARG; }
+    SPMV_TRY(check_csr(A));
+    if (A->n_rows != A->n_cols) { set_error("partition_colmap needs a square matrix"); return SPMV_ERR_INVALID_ARG; }
+    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    return colmap_impl(ctx, A, splits, nparts, as_stream(stream), colmap_out, slot);
+}
+
+spmv_status spmv_slice_remap_colmap(spmv_ctx *ctx, const spmv_csr *A, const int64_t *splits, int nparts, int part,
+                                    const int32_t *colmap, void *stream, int32_t *rp_out, int32_t *col_out,
+                                    void *val_out) {
+    if (!ctx || !splits || nparts <= 0 || part < 0 || part >= nparts || !rp_out || !colmap) {
+        set_error("bad args");
+        return SPMV_ERR_INVALID_ARG;
+    }
+    SPMV_TRY(check_csr(A));
+    if (A->n_rows != A->n_cols) { set_error("slice_remap needs a square matrix"); return SPMV_ERR_INVALID_ARG; }
+    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    return slice_remap_colmap_impl(ctx, A, splits, nparts, part, colmap, as_stream(stream), rp_out, col_out, val_out);
+}
+
+spmv_status spmv_colmap_pack_index(spmv_ctx *ctx, const int32_t *colmap, const int64_t *splits, int nparts, int part,
+                                   int64_t slot, void *stream, int32_t *idx_out, int64_t *count) {
+    if (!ctx || !colmap || !splits || nparts <= 0 || part < 0 || part >= nparts || !count || slot < 0) {
+        set_error("bad args");
+        return SPMV_ERR_INVALID_ARG;
+    }
+    if (splits[part + 1] > splits[part] && !idx_out) { set_error("NULL idx_out"); return SPMV_ERR_INVALID_ARG; }
+    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    return pack_index_impl(ctx, colmap, splits, nparts, part, slot, as_stream(stream), idx_out, count);
+}
+
+spmv_status spmv_gather(spmv_ctx *ctx, spmv_dtype dtype, const void *src, const int32_t *idx, int64_t n, void *dst,
+                        void *stream) {
+    if (!ctx || n < 0 || (n > 0 && (!src || !idx || !dst))) { set_error("bad args"); return SPMV_ERR_INVALID_ARG; }
+    if (dtype != SPMV_F32 && dtype != SPMV_F64) { set_error("bad dtype"); return SPMV_ERR_INVALID_ARG; }
+    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    return gather_impl(ctx, dtype, src, idx, n, dst, as_stream(stream));
+}
+
 }  // extern "C"

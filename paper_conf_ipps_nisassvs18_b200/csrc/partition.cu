@@ -6,6 +6,7 @@
 #include <vector>
 
 #include "internal.h"
+#include "scan.h"
 
 namespace spmv {
 
@@ -66,7 +67,139 @@ spmv_status check_splits(const spmv_csr *A, const int64_t *sp, int nparts) {
     return SPMV_OK;
 }
 
+// ---- compressed exchange
+__global__ void k_mark_used(const int *col, int64_t nnz, unsigned char *used) {
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nnz; k += (int64_t)gridDim.x * blockDim.x)
+        used[__ldg(col + k)] = 1;                 // benign race: every writer stores 1
+}
+__global__ void k_used_to_i64(const unsigned char *used, int64_t n, int64_t *out) {
+    for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
+        out[j] = used[j];
+}
+__global__ void k_colmap(const unsigned char *used, const int64_t *prefix, int64_t n, Splits sp, int *colmap) {
+    for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+        if (!used[j]) { colmap[j] = -1; continue; }
+        int lo = 0, hi = sp.nparts - 1;           // owner = last k with s[k] <= j
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (sp.s[mid] <= j) lo = mid; else hi = mid - 1;
+        }
+        colmap[j] = (int)(lo * sp.slot + (prefix[j] - prefix[sp.s[lo]]));
+    }
+}
+__global__ void k_remap_colmap(const int *col, int64_t k0, int64_t cnt, const int *colmap, int *out) {
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < cnt; k += (int64_t)gridDim.x * blockDim.x)
+        out[k] = colmap[col[k0 + k]];
+}
+__global__ void k_pack_index(const int *colmap, int64_t r0, int64_t r1, int64_t base, int *idx,
+                             unsigned long long *count) {
+    for (int64_t j = r0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < r1; j += (int64_t)gridDim.x * blockDim.x) {
+        const int c = colmap[j];
+        if (c >= 0) {
+            idx[c - base] = (int)(j - r0);
+            atomicAdd(count, 1ull);
+        }
+    }
+}
+template <typename V>
+__global__ void k_gather(const V *src, const int *idx, int64_t n, V *dst) {
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x)
+        dst[q] = src[__ldg(idx + q)];
+}
+
+int blocks_for(const spmv_ctx *ctx, int64_t n) {
+    return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div<int64_t>(n, 256), (int64_t)ctx->sm_count * 16));
+}
+
 }  // namespace
+
+spmv_status colmap_impl(spmv_ctx *ctx, const spmv_csr *A, const int64_t *sp, int nparts, cudaStream_t s,
+                        int32_t *colmap, int64_t *slot) {
+    SPMV_TRY(check_splits(A, sp, nparts));
+    const int64_t n = A->n_cols;
+    Scratch used(ctx, s), u64(ctx, s), prefix(ctx, s);
+    SPMV_TRY(used.alloc(std::max<int64_t>(n, 1)));
+    SPMV_TRY(u64.alloc(std::max<int64_t>(n, 1) * 8));
+    SPMV_TRY(prefix.alloc((n + 1) * 8));
+    SPMV_CUDA_TRY(cudaMemsetAsync(used.p, 0, std::max<int64_t>(n, 1), s));
+    if (A->nnz) {
+        k_mark_used<<<blocks_for(ctx, A->nnz), 256, 0, s>>>(A->col_idx, A->nnz, used.as<unsigned char>());
+        SPMV_LAUNCH_CHECK();
+    }
+    if (n) {
+        k_used_to_i64<<<blocks_for(ctx, n), 256, 0, s>>>(used.as<unsigned char>(), n, u64.as<int64_t>());
+        SPMV_LAUNCH_CHECK();
+    }
+    SPMV_TRY(exclusive_scan_i64(ctx, u64.as<int64_t>(), prefix.as<int64_t>(), n, s));
+    std::vector<int64_t> at(nparts + 1);
+    for (int k = 0; k <= nparts; ++k)
+        SPMV_CUDA_TRY(cudaMemcpyAsync(&at[k], prefix.as<int64_t>() + sp[k], 8, cudaMemcpyDeviceToHost, s));
+    SPMV_CUDA_TRY(cudaStreamSynchronize(s));
+    int64_t S = 0;
+    for (int k = 0; k < nparts; ++k) S = std::max(S, at[k + 1] - at[k]);
+    if ((int64_t)nparts * S > (int64_t)INT32_MAX) { set_error("compressed slots exceed int32"); return SPMV_ERR_SIZE; }
+    Splits spl{};
+    for (int k = 0; k <= nparts; ++k) spl.s[k] = sp[k];
+    spl.nparts = nparts;
+    spl.slot = S;
+    if (n) {
+        k_colmap<<<blocks_for(ctx, n), 256, 0, s>>>(used.as<unsigned char>(), prefix.as<int64_t>(), n, spl, colmap);
+        SPMV_LAUNCH_CHECK();
+    }
+    *slot = S;
+    return SPMV_OK;
+}
+
+spmv_status slice_remap_colmap_impl(spmv_ctx *ctx, const spmv_csr *A, const int64_t *sp, int nparts, int part,
+                                    const int32_t *colmap, cudaStream_t s, int32_t *rp_out, int32_t *col_out,
+                                    void *val_out) {
+    int64_t rows = 0, nnz = 0, S = 0;
+    SPMV_TRY(slice_size_impl(ctx, A, sp, nparts, part, s, &rows, &nnz, &S));
+    if (nnz > INT32_MAX) { set_error("shard exceeds int32 indices"); return SPMV_ERR_SIZE; }
+    if (nnz > 0 && (!col_out || !val_out)) { set_error("NULL col/val out"); return SPMV_ERR_INVALID_ARG; }
+    int64_t k0 = 0;
+    SPMV_TRY(rp_at(A, sp[part], s, &k0));
+    if (A->ptr_type == SPMV_I32)
+        k_rebase<int><<<blocks_for(ctx, rows + 1), 256, 0, s>>>((const int *)A->row_ptr, sp[part], rows, rp_out);
+    else
+        k_rebase<int64_t><<<blocks_for(ctx, rows + 1), 256, 0, s>>>((const int64_t *)A->row_ptr, sp[part], rows, rp_out);
+    SPMV_LAUNCH_CHECK();
+    if (nnz > 0) {
+        k_remap_colmap<<<blocks_for(ctx, nnz), 256, 0, s>>>(A->col_idx, k0, nnz, colmap, col_out);
+        SPMV_LAUNCH_CHECK();
+        const size_t V = A->dtype == SPMV_F64 ? 8 : 4;
+        SPMV_CUDA_TRY(cudaMemcpyAsync(val_out, (const char *)A->vals + k0 * V, nnz * V, cudaMemcpyDeviceToDevice, s));
+    }
+    return SPMV_OK;
+}
+
+spmv_status pack_index_impl(spmv_ctx *ctx, const int32_t *colmap, const int64_t *sp, int nparts, int part,
+                            int64_t slot, cudaStream_t s, int32_t *idx, int64_t *count) {
+    Scratch cnt(ctx, s);
+    SPMV_TRY(cnt.alloc(8));
+    SPMV_CUDA_TRY(cudaMemsetAsync(cnt.p, 0, 8, s));
+    const int64_t r0 = sp[part], r1 = sp[part + 1];
+    if (r1 > r0) {
+        k_pack_index<<<blocks_for(ctx, r1 - r0), 256, 0, s>>>(colmap, r0, r1, (int64_t)part * slot, idx,
+                                                             cnt.as<unsigned long long>());
+        SPMV_LAUNCH_CHECK();
+    }
+    unsigned long long c = 0;
+    SPMV_CUDA_TRY(cudaMemcpyAsync(&c, cnt.p, 8, cudaMemcpyDeviceToHost, s));
+    SPMV_CUDA_TRY(cudaStreamSynchronize(s));
+    *count = (int64_t)c;
+    (void)nparts;
+    return SPMV_OK;
+}
+
+spmv_status gather_impl(spmv_ctx *ctx, spmv_dtype dt, const void *src, const int32_t *idx, int64_t n, void *dst,
+                        cudaStream_t s) {
+    if (n <= 0) return SPMV_OK;
+    if (dt == SPMV_F64) k_gather<double><<<blocks_for(ctx, n), 256, 0, s>>>((const double *)src, idx, n, (double *)dst);
+    else k_gather<float><<<blocks_for(ctx, n), 256, 0, s>>>((const float *)src, idx, n, (float *)dst);
+    SPMV_LAUNCH_CHECK();
+    return SPMV_OK;
+}
 
 spmv_status partition_impl(spmv_ctx *ctx, const spmv_csr *A, int nparts, cudaStream_t s, int64_t *splits) {
     Scratch d(ctx, s);

@@ -22,7 +22,8 @@ import numpy as np
 import torch
 import torch.distributed as dist
 
-from .spmv import CSR, convert, partition, slice_remap
+from .spmv import (CSR, convert, partition, slice_remap, spmv_colmap_pack_index, spmv_gather,
+                   spmv_partition_colmap, spmv_slice_remap_colmap)
 
 
 @dataclass
@@ -88,9 +89,11 @@ class DistSpMV:
 
     ``A`` is the full matrix on this rank's GPU (every rank builds the same one; the
     partition kernel is deterministic and rank 0's splits are broadcast and checked).
+    ``compress=True`` exchanges only the columns some row references:
+    slots of S' = max referenced columns per part, packed every step by ``spmv_gather``.
     """
 
-    def __init__(self, A: CSR, fmt: str = "csr5", group=None, **convert_opts):
+    def __init__(self, A: CSR, fmt: str = "csr5", group=None, compress: bool = False, **convert_opts):
         if A.n_rows != A.n_cols:
             raise ValueError("DistSpMV needs a square matrix (x is owned like y)")
         self.group = group
@@ -103,11 +106,19 @@ class DistSpMV:
         if not torch.equal(t, t0):
             raise RuntimeError("ranks disagree on the row partition (different matrices?)")
         self.layout = ShardLayout(splits, rank)
-        self.shard, S = slice_remap(A, splits, rank)
-        assert S == self.layout.S
+        self.compress = compress
+        dev = A.row_ptr.device
+        if compress:
+            colmap, S = spmv_partition_colmap(A, splits)
+            self.shard = spmv_slice_remap_colmap(A, splits, rank, colmap, S)
+            self.pack_idx = spmv_colmap_pack_index(colmap, splits, rank, S)
+        else:
+            self.shard, S = slice_remap(A, splits, rank)
+            assert S == self.layout.S
+            self.pack_idx = None
+        self.slot = S
         self.handle = convert(self.shard, fmt, **convert_opts)
         self.dtype = A.val.dtype
-        dev = A.row_ptr.device
         self.x_slot = torch.zeros(S, dtype=self.dtype, device=dev)
         self.x_gathered = torch.zeros(P * S, dtype=self.dtype, device=dev)
 
@@ -115,9 +126,16 @@ class DistSpMV:
     def rows(self) -> int:
         return self.layout.rows
 
+    def exchange_bytes(self) -> int:
+        """Bytes each rank receives per step."""
+        return (self.layout.P - 1) * self.slot * self.x_slot.element_size()
+
     def set_x(self, x_local: torch.Tensor):
-        """Stage this rank's x slice (length rows) into its padded slot."""
-        self.layout.pack_x(x_local, out=self.x_slot)
+        """Stage this rank's x slice (length rows) into its padded / compressed slot."""
+        if self.compress:
+            spmv_gather(x_local, self.pack_idx, self.x_slot)
+        else:
+            self.layout.pack_x(x_local, out=self.x_slot)
 
     def exchange(self):
         """All-gather the x slots (the one collective of a step)."""

@@ -124,6 +124,13 @@ def lib():
                                           C.POINTER(C.c_int64), C.POINTER(C.c_int64), C.POINTER(C.c_int64)]),
             "spmv_slice_remap": (C.c_int, [_P, C.POINTER(spmv_csr), C.POINTER(C.c_int64), C.c_int, C.c_int, _P,
                                            _P, _P, _P]),
+            "spmv_partition_colmap": (C.c_int, [_P, C.POINTER(spmv_csr), C.POINTER(C.c_int64), C.c_int, _P, _P,
+                                                C.POINTER(C.c_int64)]),
+            "spmv_slice_remap_colmap": (C.c_int, [_P, C.POINTER(spmv_csr), C.POINTER(C.c_int64), C.c_int, C.c_int,
+                                                  _P, _P, _P, _P, _P]),
+            "spmv_colmap_pack_index": (C.c_int, [_P, _P, C.POINTER(C.c_int64), C.c_int, C.c_int, C.c_int64, _P, _P,
+                                                 C.POINTER(C.c_int64)]),
+            "spmv_gather": (C.c_int, [_P, C.c_int, _P, _P, C.c_int64, _P, _P]),
             "spmv_status_str": (C.c_char_p, [C.c_int]),
             "spmv_last_error": (C.c_char_p, []),
         }
@@ -302,6 +309,66 @@ def spmv_slice_remap(A: CSR, splits, part: int, stream=None):
 
 
 slice_remap = spmv_slice_remap
+
+
+def _splits_c(splits):
+    sp = np.ascontiguousarray(splits, dtype=np.int64)
+    return sp, (C.c_int64 * sp.size)(*sp.tolist())
+
+
+def spmv_partition_colmap(A: CSR, splits, stream=None):
+    """Compressed exchange map: int32 device colmap[n_cols] and slot S'."""
+    ctx = context(A.row_ptr.device.index)
+    sp, csp = _splits_c(splits)
+    colmap = torch.empty(A.n_cols, dtype=torch.int32, device=A.row_ptr.device)
+    slot = C.c_int64()
+    a = A.as_c()
+    _check(lib().spmv_partition_colmap(ctx.ptr, C.byref(a), csp, sp.size - 1, _stream_ptr(stream),
+                                       colmap.data_ptr() if A.n_cols else None, C.byref(slot)))
+    return colmap, slot.value
+
+
+def spmv_slice_remap_colmap(A: CSR, splits, part: int, colmap: torch.Tensor, slot: int, stream=None) -> CSR:
+    """Shard `part` with columns mapped through the compressed colmap."""
+    ctx = context(A.row_ptr.device.index)
+    sp, csp = _splits_c(splits)
+    P = sp.size - 1
+    a = A.as_c()
+    rows, nnz, dslot = C.c_int64(), C.c_int64(), C.c_int64()
+    st = _stream_ptr(stream)
+    _check(lib().spmv_slice_size(ctx.ptr, C.byref(a), csp, P, int(part), st, C.byref(rows), C.byref(nnz),
+                                 C.byref(dslot)))
+    dev = A.row_ptr.device
+    rp = torch.empty(rows.value + 1, dtype=torch.int32, device=dev)
+    col = torch.empty(nnz.value, dtype=torch.int32, device=dev)
+    val = torch.empty(nnz.value, dtype=A.val.dtype, device=dev)
+    _check(lib().spmv_slice_remap_colmap(ctx.ptr, C.byref(a), csp, P, int(part), colmap.data_ptr(), st,
+                                         rp.data_ptr(), col.data_ptr() if nnz.value else None,
+                                         val.data_ptr() if nnz.value else None))
+    return CSR(rp, col, val, (rows.value, P * slot))
+
+
+def spmv_colmap_pack_index(colmap: torch.Tensor, splits, part: int, slot: int, stream=None) -> torch.Tensor:
+    """Local positions (int32 device) of part `part`'s exchanged columns, in slot order."""
+    ctx = context(colmap.device.index)
+    sp, csp = _splits_c(splits)
+    rows = int(sp[part + 1] - sp[part])
+    idx = torch.empty(max(rows, 1), dtype=torch.int32, device=colmap.device)
+    cnt = C.c_int64()
+    _check(lib().spmv_colmap_pack_index(ctx.ptr, colmap.data_ptr(), csp, sp.size - 1, int(part), int(slot),
+                                        _stream_ptr(stream), idx.data_ptr(), C.byref(cnt)))
+    return idx[: cnt.value]
+
+
+def spmv_gather(src: torch.Tensor, idx: torch.Tensor, dst: torch.Tensor, stream=None):
+    """dst[q] = src[idx[q]] on the GPU (the per-step compressed-slot packing)."""
+    ctx = context(src.device.index)
+    n = idx.numel()
+    dt = 1 if src.dtype == torch.float64 else 0
+    _check(lib().spmv_gather(ctx.ptr, dt, src.data_ptr() if src.numel() else None,
+                             idx.data_ptr() if n else None, n, dst.data_ptr() if dst.numel() else None,
+                             _stream_ptr(stream)))
+    return dst
 
 
 # ----------------------------------------------------------------- handle

@@ -25,7 +25,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, case, q):
+def _worker(rank, world, port, case, q, compress=False):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -43,17 +43,28 @@ def _worker(rank, world, port, case, q):
         y = matgen.vector(A.n_rows, 32, 2)
         splits = oracle.partition(A, world)
         lay = ShardLayout(splits, rank)
-        # every rank holds only its x slice; the gathered vector is built by the collective
-        slot = lay.pack_x(torch.from_numpy(x[lay.r0:lay.r1].copy()))
-        gathered = torch.zeros(world * lay.S, dtype=torch.float64)
-        all_gather_slots(gathered, slot)
-        rp, col, val = oracle.slice_remap(A, splits, rank)
-        shard = matgen.HostCSR(rp, col, val, lay.rows, world * lay.S)
+        if compress:
+            # only columns some row references are exchanged
+            cm, S = oracle.partition_colmap(A, splits)
+            js = np.nonzero(cm[lay.r0:lay.r1] >= 0)[0]
+            slot = torch.zeros(S, dtype=torch.float64)
+            slot[: js.size] = torch.from_numpy(x[lay.r0 + js].copy())
+            gathered = torch.zeros(world * S, dtype=torch.float64)
+            all_gather_slots(gathered, slot)
+            rp, col, val = oracle.slice_remap_colmap(A, splits, rank, cm)
+            shard = matgen.HostCSR(rp, col, val, lay.rows, world * S)
+        else:
+            # every rank holds only its x slice; the gathered vector is built by the collective
+            slot = lay.pack_x(torch.from_numpy(x[lay.r0:lay.r1].copy()))
+            gathered = torch.zeros(world * lay.S, dtype=torch.float64)
+            all_gather_slots(gathered, slot)
+            rp, col, val = oracle.slice_remap(A, splits, rank)
+            shard = matgen.HostCSR(rp, col, val, lay.rows, world * lay.S)
         y_local = oracle.spmv_csr(shard, gathered.numpy(), 1.25, -0.5, y[lay.r0:lay.r1])
         # slot_of agrees with the remap
         for k in range(0, A.nnz, max(1, A.nnz // 50)):
             r = int(np.searchsorted(A.row_ptr, k, side="right")) - 1
-            if lay.r0 <= r < lay.r1:
+            if lay.r0 <= r < lay.r1 and not compress:
                 assert col[k - A.row_ptr[lay.r0]] == lay.slot_of(int(A.col[k]))
         # assemble y for the check (padded equal-count gather)
         yslot = lay.pack_x(torch.from_numpy(y_local))
@@ -68,13 +79,16 @@ def _worker(rank, world, port, case, q):
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("compress", [False, True])
 @pytest.mark.parametrize("world", [2, 3])
 @pytest.mark.parametrize("case", ["rmat", "lap", "ragged"])
-def test_partitioned_spmv_gloo(world, case):
+def test_partitioned_spmv_gloo(world, case, compress):
+    if compress and case == "lap":
+        pytest.skip("every column of the Laplacian is referenced")
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, case, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, case, q, compress)) for r in range(world)]
     for p in procs:
         p.start()
     for p in procs:

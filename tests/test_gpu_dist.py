@@ -72,3 +72,71 @@ def test_distspmv_nccl_world1(sp):
         assert oracle.check_tolerance(full, ref, bound, 1e-12)[0]
     finally:
         dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("P", [1, 2, 4, 8])
+@pytest.mark.parametrize("case", ["rmat13", "empty_cols"])
+def test_compressed_exchange(sp, case, P):
+    """colmap / compressed remap / pack index bit-exact against the oracle, and the
+    compressed virtual partition reproduces the product."""
+    from paper_conf_ipps_nisassvs18_b200.spmv import (spmv_colmap_pack_index, spmv_gather,
+                                                       spmv_partition_colmap, spmv_slice_remap_colmap)
+    if case == "rmat13":
+        A = matgen.rmat(13, seed=47)
+    else:
+        lens = np.random.default_rng(3).integers(0, 6, 4000)
+        A = matgen.from_lengths(lens, 4000, seed=48)
+        keep = A.col % 3 != 0                                  # a third of the columns never used
+        rows = np.repeat(np.arange(A.n_rows), np.diff(A.row_ptr))[keep]
+        rp = np.zeros(A.n_rows + 1, np.int64)
+        np.add.at(rp, rows + 1, 1)
+        A = matgen.HostCSR(np.cumsum(rp), A.col[keep].copy(), A.val[keep].copy(), A.n_rows, A.n_cols)
+    x = matgen.vector(A.n_cols, 47, 1)
+    y = matgen.vector(A.n_rows, 47, 2)
+    ref, bound = oracle.spmv_csr(A, x, 1.0, -1.0, y, with_bound=True)
+    dA = sp.CSR.from_host(A)
+    splits = sp.partition(dA, P)
+    cm_o, S_o = oracle.partition_colmap(A, splits)
+    cm, S = spmv_partition_colmap(dA, splits)
+    assert S == S_o and np.array_equal(cm.cpu().numpy(), cm_o)
+    xd = torch.from_numpy(x).cuda()
+    xg = torch.zeros(P * S, dtype=torch.float64, device="cuda")
+    for k in range(P):
+        idx = spmv_colmap_pack_index(cm, splits, k, S)
+        exp_idx = np.nonzero(cm_o[splits[k]:splits[k + 1]] >= 0)[0]
+        assert np.array_equal(idx.cpu().numpy(), exp_idx)
+        spmv_gather(xd[int(splits[k]):int(splits[k + 1])], idx, xg[k * S:(k + 1) * S])
+    out = np.empty(A.n_rows)
+    for k in range(P):
+        shard = spmv_slice_remap_colmap(dA, splits, k, cm, S)
+        rp, col, val = oracle.slice_remap_colmap(A, splits, k, cm_o)
+        assert np.array_equal(shard.col.cpu().numpy(), col)
+        assert np.array_equal(shard.row_ptr.cpu().numpy().astype(np.int64), rp)
+        h = sp.convert(shard, "csr5")
+        yl = torch.from_numpy(y[splits[k]:splits[k + 1]].copy()).cuda()
+        h.run(1.0, xg, -1.0, yl)
+        out[splits[k]:splits[k + 1]] = yl.cpu().numpy()
+    assert oracle.check_tolerance(out, ref, bound, 1e-12)[0]
+
+
+def test_distspmv_nccl_world1_compressed(sp):
+    import torch.distributed as dist
+    from paper_conf_ipps_nisassvs18_b200.dist import DistSpMV
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK="0", WORLD_SIZE="1")
+    dist.init_process_group("nccl", device_id=torch.device("cuda", 0))
+    try:
+        A = matgen.rmat(12, seed=44)
+        x = matgen.vector(A.n_cols, 44, 1)
+        y = matgen.vector(A.n_rows, 44, 2)
+        ref, bound = oracle.spmv_csr(A, x, 1.0, 1.0, y, with_bound=True)
+        D = DistSpMV(sp.CSR.from_host(A), "merge", compress=True)
+        assert D.slot < A.n_cols                               # R-MAT has empty columns
+        yl = torch.from_numpy(y.copy()).cuda()
+        D.run(1.0, 1.0, yl, x_local=torch.from_numpy(x).cuda())
+        assert oracle.check_tolerance(yl.cpu().numpy(), ref, bound, 1e-12)[0]
+    finally:
+        dist.destroy_process_group()
