@@ -138,6 +138,8 @@ typedef struct {
                               64 MiB)))                                                    */
     int alias_input;       /* 1 = COO/CSR handles reference the caller's col/vals (caller
                               keeps them alive and unchanged); MERGE/CSR5/ELL/HYB copy     */
+    int index64;           /* 1 = int64 row pointers/offsets inside the handle even when
+                              nnz <= INT32_MAX (exercises the > 2^31-nonzero path, A17)   */
 } spmv_convert_opts;
 
 /* Fill `opts` with the defaults (all rules as above). */

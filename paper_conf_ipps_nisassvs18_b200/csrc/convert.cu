@@ -472,7 +472,7 @@ spmv_status convert_impl(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, cons
         set_error("matrix is not canonical (flags " + std::to_string(fs.bad) + ")");
         return SPMV_ERR_NOT_CANONICAL;
     }
-    const bool i64 = A->nnz > INT32_MAX;
+    const bool i64 = A->nnz > INT32_MAX || o->index64;
     if (A->dtype == SPMV_F64) {
         return i64 ? convert_t<int64_t, double>(ctx, fmt, A, o, s, h, fs, cusp)
                    : convert_t<int, double>(ctx, fmt, A, o, s, h, fs, cusp);

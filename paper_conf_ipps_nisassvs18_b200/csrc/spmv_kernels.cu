@@ -95,6 +95,9 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
             b[u] = i + 1 < R ? nx : rp_hi;
             if (base + i >= n) { a[u] = 0; b[u] = 0; }
         }
+        // the y value this lane will write (writer lane sub == u of group g: row u*G + g)
+        const int64_t my_row = base + (int64_t)sub * G + g;
+        const double yv = (!B0 && sub < U && my_row < n) ? (double)y[my_row] : 0.0;
         // first W elements of every row, all loads issued together
         int c0[U];
         V v0[U];
@@ -154,13 +157,10 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
                 if (lane == writer) mine += part;
             }
         }
-        if (sub < U) {
-            const int64_t r = base + sub * G + g;
-            if (r < n) {
-                double o = alpha * mine;
-                if (!B0) o = fma(beta, (double)y[r], o);
-                y[r] = (V)o;
-            }
+        if (sub < U && my_row < n) {
+            double o = alpha * mine;
+            if (!B0) o = fma(beta, yv, o);
+            y[my_row] = (V)o;
         }
     }
 }

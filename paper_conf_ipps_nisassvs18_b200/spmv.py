@@ -71,7 +71,7 @@ PAPER_FEATURES = ("n_rows", "n_cols", "nnz_tot", "nnz_mu", "nnz_frac",          
 class spmv_convert_opts(C.Structure):
     _fields_ = [("hyb_rule", C.c_int), ("hyb_width", C.c_int64), ("csr5_sigma", C.c_int),
                 ("merge_items", C.c_int), ("vector_width", C.c_int), ("max_bytes", C.c_size_t),
-                ("alias_input", C.c_int)]
+                ("alias_input", C.c_int), ("index64", C.c_int)]
 
 
 class spmv_handle_info(C.Structure):

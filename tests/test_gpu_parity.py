@@ -417,3 +417,33 @@ def _lap_ref(A, x, y0):
     if "lapref" not in _BIG:
         _BIG["lapref"] = oracle.spmv_csr(A, x, 1.0, 1.0, y0, with_bound=True)
     return _BIG["lapref"]
+
+
+I64_CASES = ["rmat15", "empty_runs", "long_row", "tile_bounds", "u2048", "nnz0_rows5", "rect_7x3"]
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32], ids=["f64", "f32"])
+@pytest.mark.parametrize("fmt", ALL_FORMATS)
+@pytest.mark.parametrize("name", I64_CASES)
+def test_index64_path(sp, name, fmt, dtype):
+    """A17: handles with int64 row pointers/offsets (the > 2^31-nonzero path of configs[4]),
+    forced on small matrices with convert option index64=1."""
+    A = case(name, KIND[dtype])
+    dA = to_dev(sp, A, dtype)
+    if expected_infeasible(A, fmt, dtype):
+        pytest.skip("infeasible (A4)")
+    x = matgen.vector(A.n_cols, 88, 1, KIND[dtype])
+    y0 = matgen.vector(A.n_rows, 88, 2, KIND[dtype])
+    ref, bound = oracle.spmv_csr(A, x, 1.5, -0.5, y0, with_bound=True)
+    h, out = run_format(sp, A, dA, fmt, dtype, 1.5, -0.5, x, y0, index64=1)
+    if fmt in ("csr", "csr_scalar", "merge", "csr5"):
+        assert h.info()["ptr_type"] == 1
+    ok, ratio, nbad = oracle.check_tolerance(out, ref, bound, TOL[dtype])
+    assert ok, (nbad, ratio)
+    if fmt == "merge":
+        cr, cn = oracle.merge_coords(A, h.info()["merge_items"])
+        assert np.array_equal(h.export("merge_coord_nz"), cn)
+    if fmt == "csr5":
+        e = oracle.csr5_encode(A, val_bytes=8 if dtype == torch.float64 else 4)
+        assert np.array_equal(h.export("csr5_tile_desc"), e["tile_desc"])
+        assert np.array_equal(h.export("row_ptr"), A.row_ptr)
