@@ -524,8 +524,8 @@ template <int N> struct ShiftLoad<int, N> {
     static __device__ __forceinline__ void load(const int *p, int (&v)[N], uint64_t pol) { shift_load4<int, int4, N>(p, v, pol); }
 };
 
-template <typename V, typename IT, bool B0, int LI>
-__global__ void __launch_bounds__(kT, LI == 4 ? 6 : kMinBlocks)
+template <typename V, typename IT, bool B0, int LI, int MB = kMinBlocks>
+__global__ void __launch_bounds__(kT, MB)
 k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
         const int64_t *__restrict__ crow, const int64_t *__restrict__ cnz, int64_t n_tiles, int64_t n_rows,
         const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
@@ -922,10 +922,11 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
         const unsigned g = (unsigned)ceil_div<int64_t>(h->merge_tiles, kT / 32);
         const int64_t *cr = (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_ROW].p;
         const int64_t *cz = (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_NZ].p;
+        // 4 CTAs/SM (<= 64 registers) measured best for both tile sizes' siblings (3, 5, 6 slower)
         if (h->merge_T == 128)
-            k_merge<V, IT, B0, 4><<<g, kT, 0, s>>>(rp, col, val, cr, cz, h->merge_tiles, n, x, y, alpha, beta, crow, cval);
+            k_merge<V, IT, B0, 4, 6><<<g, kT, 0, s>>>(rp, col, val, cr, cz, h->merge_tiles, n, x, y, alpha, beta, crow, cval);
         else
-            k_merge<V, IT, B0, 8><<<g, kT, 0, s>>>(rp, col, val, cr, cz, h->merge_tiles, n, x, y, alpha, beta, crow, cval);
+            k_merge<V, IT, B0, 8, 4><<<g, kT, 0, s>>>(rp, col, val, cr, cz, h->merge_tiles, n, x, y, alpha, beta, crow, cval);
     }
         SPMV_LAUNCH_CHECK();
         return launch_fixup<V>(h, y, alpha, s);
