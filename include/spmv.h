@@ -263,6 +263,19 @@ spmv_status spmv_colmap_pack_index(spmv_ctx *ctx, const int32_t *colmap, const i
                                    int nparts, int part, int64_t slot, void *stream, int32_t *idx_out,
                                    int64_t *count);
 
+/* Overlap of the exchange with compute: shard `part` split by column
+ * ownership.  which = 0: the OWN block -- columns in [splits[part], splits[part+1]), remapped
+ * to j - splits[part] (they index the rank's own x slice, available before the exchange);
+ * which = 1: the FOREIGN block -- all other columns, remapped to gathered-x slots (dense layout
+ * when colmap == NULL, else through colmap with slot layout of spmv_partition_colmap).
+ * Both blocks cover the same rows [splits[part], splits[part+1]).
+ * row_ptr_out[rows+1] (DEVICE int32) is always written and *nnz_out (host) receives the
+ * block's nonzero count; col_out/vals_out (DEVICE) may be NULL for this sizing call, else
+ * they receive the block.  Blocks on `stream`. */
+spmv_status spmv_slice_split(spmv_ctx *ctx, const spmv_csr *A, const int64_t *row_splits_host, int nparts,
+                             int part, const int32_t *colmap, int which, void *stream, int32_t *row_ptr_out,
+                             int32_t *col_out, void *vals_out, int64_t *nnz_out);
+
 /* dst[q] = src[idx[q]] for q < n (DEVICE arrays of `dtype`): the per-step packing of a
  * rank's x slice into its compressed slot.  Asynchronous. */
 spmv_status spmv_gather(spmv_ctx *ctx, spmv_dtype dtype, const void *src, const int32_t *idx, int64_t n,

@@ -90,6 +90,7 @@ def lib():
             "ora_slice_remap": (C.c_int, [_i64, _p, _p, _p, _p, C.c_int, C.c_int, _p, _p, _p]),
             "ora_partition_colmap": (_i64, [_i64, _p, _p, _p, C.c_int, _p]),
             "ora_slice_remap_colmap": (C.c_int, [_i64, _p, _p, _p, _p, C.c_int, _p, _p, _p, _p]),
+            "ora_slice_split": (_i64, [_i64, _p, _p, _p, _p, C.c_int, C.c_int, _p, C.c_int, _p, _p, _p]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -323,6 +324,20 @@ def slice_remap_colmap(A, splits, part, colmap):
     rc = lib().ora_slice_remap_colmap(A.n_rows, _ptr(A.row_ptr), _ptr(A.col), _ptr(A.val), _ptr(s), int(part),
                                       _ptr(cm), _ptr(rp), _ptr(col), _ptr(val))
     assert rc == 0
+    return rp, col, val
+
+
+def slice_split(A, splits, part, which, colmap=None):
+    """Own (which=0) / foreign (which=1) block of shard `part`."""
+    A = CSR.of(A)
+    s = _c(splits, np.int64)
+    cm = _c(colmap, np.int32) if colmap is not None else None
+    r0, r1 = int(s[part]), int(s[part + 1])
+    n = lib().ora_slice_split(A.n_rows, _ptr(A.row_ptr), _ptr(A.col), _ptr(A.val), _ptr(s), s.size - 1, int(part),
+                              _ptr(cm) if cm is not None else None, int(which), None, None, None)
+    rp, col, val = _buf(r1 - r0 + 1, np.int64), _buf(n, np.int32), _buf(n, np.float64)
+    lib().ora_slice_split(A.n_rows, _ptr(A.row_ptr), _ptr(A.col), _ptr(A.val), _ptr(s), s.size - 1, int(part),
+                          _ptr(cm) if cm is not None else None, int(which), _ptr(rp), _ptr(col), _ptr(val))
     return rp, col, val
 
 

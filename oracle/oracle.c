@@ -574,3 +574,34 @@ int ora_slice_remap_colmap(int64_t n_rows, const int64_t *row_ptr, const int32_t
     }
     return 0;
 }
+
+/* Own / foreign split of a shard: plain row-by-row filter in stored order. */
+int64_t ora_slice_split(int64_t n_rows, const int64_t *row_ptr, const int32_t *col, const double *val,
+                        const int64_t *splits, int nparts, int part, const int32_t *colmap, int which,
+                        int64_t *out_row_ptr, int32_t *out_col, double *out_val)
+{
+    int64_t r0 = splits[part], r1 = splits[part + 1];
+    int64_t S = ora_partition_slot(splits, nparts), q = 0;
+    if (r1 > n_rows) return -1;
+    for (int64_t r = r0; r < r1; ++r) {
+        if (out_row_ptr) out_row_ptr[r - r0] = q;
+        for (int64_t k = row_ptr[r]; k < row_ptr[r + 1]; ++k) {
+            int64_t j = col[k];
+            int own = j >= r0 && j < r1;
+            if (own != (which == 0)) continue;
+            if (out_col) {
+                if (which == 0) out_col[q] = (int32_t)(j - r0);
+                else if (colmap) out_col[q] = colmap[j];
+                else {
+                    int owner = 0;
+                    while (!(splits[owner] <= j && j < splits[owner + 1])) ++owner;
+                    out_col[q] = (int32_t)(owner * S + (j - splits[owner]));
+                }
+                out_val[q] = val[k];
+            }
+            ++q;
+        }
+    }
+    if (out_row_ptr) out_row_ptr[r1 - r0] = q;
+    return q;
+}

@@ -145,6 +145,14 @@ int ora_slice_remap_colmap(int64_t n_rows, const int64_t *row_ptr, const int32_t
                            const double *val, const int64_t *splits, int part, const int32_t *colmap,
                            int64_t *out_row_ptr, int32_t *out_col, double *out_val);
 
+/* Own / foreign split of shard `part`: which = 0 keeps columns in the
+ * part's own row range, remapped to j - splits[part]; which = 1 keeps the others,
+ * remapped to the dense slot layout (colmap == NULL) or through colmap.  Returns the
+ * block's nonzero count; out_* may be NULL to size only. */
+int64_t ora_slice_split(int64_t n_rows, const int64_t *row_ptr, const int32_t *col, const double *val,
+                        const int64_t *splits, int nparts, int part, const int32_t *colmap, int which,
+                        int64_t *out_row_ptr, int32_t *out_col, double *out_val);
+
 #ifdef __cplusplus
 }
 #endif

@@ -3,9 +3,21 @@
 #include <new>
 #include <string>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "internal.h"
 
 namespace spmv {
+
+// NVTX ranges (SURVEY §5 tracing): visible in Nsight Systems / ncu --nvtx, free otherwise
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
+static const char *kRunNames[] = {"spmv_run:coo", "spmv_run:ell", "spmv_run:csr", "spmv_run:hyb",
+                                  "spmv_run:merge", "spmv_run:csr5", "spmv_run:csr_scalar"};
+static const char *kConvNames[] = {"spmv_convert:coo", "spmv_convert:ell", "spmv_convert:csr", "spmv_convert:hyb",
+                                   "spmv_convert:merge", "spmv_convert:csr5", "spmv_convert:csr_scalar"};
 
 static thread_local std::string g_err;
 void set_error(const std::string &msg) { g_err = msg; }
@@ -122,6 +134,7 @@ spmv_status spmv_device_info(const spmv_ctx *ctx, int *sm_count, int64_t *l2_byt
 }
 
 spmv_status spmv_features(spmv_ctx *ctx, const spmv_csr *A, void *stream, spmv_features_t *out) {
+    NvtxRange nv("spmv_features");
     if (!ctx || !out) { set_error("NULL ctx/out"); return SPMV_ERR_INVALID_ARG; }
     SPMV_TRY(check_csr(A));
     SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
@@ -149,6 +162,7 @@ spmv_status spmv_convert(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A,
     *out = nullptr;
     SPMV_TRY(check_csr(A));
     if ((int)fmt < 0 || (int)fmt > (int)SPMV_CSR_SCALAR) { set_error("bad format"); return SPMV_ERR_INVALID_ARG; }
+    NvtxRange nv(kConvNames[fmt]);
     spmv_convert_opts o;
     spmv_convert_opts_default(&o);
     if (opts) o = *opts;
@@ -192,6 +206,7 @@ spmv_status spmv_run(spmv_handle *h, const void *alpha, const void *x, const voi
     double a, b;
     if (h->dtype == SPMV_F64) { a = *(const double *)alpha; b = *(const double *)beta; }
     else { a = *(const float *)alpha; b = *(const float *)beta; }
+    NvtxRange nv(kRunNames[h->fmt]);
     return run_impl(h, a, b, x, y, as_stream(stream));
 }
 
@@ -294,6 +309,7 @@ spmv_status spmv_destroy(spmv_handle *h, void *stream) {
 }
 
 spmv_status spmv_partition(spmv_ctx *ctx, const spmv_csr *A, int nparts, void *stream, int64_t *splits) {
+    NvtxRange nv("spmv_partition");
     if (!ctx || !splits || nparts <= 0) { set_error("bad ctx/splits/nparts"); return SPMV_ERR_INVALID_ARG; }
     SPMV_TRY(check_csr(A));
     SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
@@ -348,6 +364,19 @@ spmv_status spmv_colmap_pack_index(spmv_ctx *ctx, const int32_t *colmap, const i
     if (splits[part + 1] > splits[part] && !idx_out) { set_error("NULL idx_out"); return SPMV_ERR_INVALID_ARG; }
     SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
     return pack_index_impl(ctx, colmap, splits, nparts, part, slot, as_stream(stream), idx_out, count);
+}
+
+spmv_status spmv_slice_split(spmv_ctx *ctx, const spmv_csr *A, const int64_t *splits, int nparts, int part,
+                             const int32_t *colmap, int which, void *stream, int32_t *rp_out, int32_t *col_out,
+                             void *val_out, int64_t *nnz_out) {
+    if (!ctx || !splits || nparts <= 0 || part < 0 || part >= nparts || !rp_out || !nnz_out || (which != 0 && which != 1)) {
+        set_error("bad args");
+        return SPMV_ERR_INVALID_ARG;
+    }
+    SPMV_TRY(check_csr(A));
+    if (A->n_rows != A->n_cols) { set_error("slice_split needs a square matrix"); return SPMV_ERR_INVALID_ARG; }
+    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    return split_impl(ctx, A, splits, nparts, part, colmap, which, as_stream(stream), rp_out, col_out, val_out, nnz_out);
 }
 
 spmv_status spmv_gather(spmv_ctx *ctx, spmv_dtype dtype, const void *src, const int32_t *idx, int64_t n, void *dst,

@@ -107,6 +107,54 @@ __global__ void k_gather(const V *src, const int *idx, int64_t n, V *dst) {
         dst[q] = src[__ldg(idx + q)];
 }
 
+// own / foreign split of a shard
+template <typename IT>
+__global__ void k_split_count(const IT *rp, const int *col, int64_t r0, int64_t rows, int64_t c0, int64_t c1,
+                              int which, int64_t *cnt) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < rows; i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t c = 0;
+        for (int64_t k = rp[r0 + i]; k < (int64_t)rp[r0 + i + 1]; ++k) {
+            const int64_t j = col[k];
+            const bool own = j >= c0 && j < c1;
+            c += (which == 0) == own;
+        }
+        cnt[i] = c;
+    }
+}
+__global__ void k_i64_to_i32(const int64_t *in, int64_t n, int *out) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = (int)in[i];
+}
+template <typename IT, typename V>
+__global__ void k_split_fill(const IT *rp, const int *col, const V *val, int64_t r0, int64_t rows, int64_t c0,
+                             int64_t c1, int which, Splits sp, const int *colmap, const int *rp_out, int *col_out,
+                             V *val_out) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < rows; i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t q = rp_out[i];
+        for (int64_t k = rp[r0 + i]; k < (int64_t)rp[r0 + i + 1]; ++k) {
+            const int64_t j = col[k];
+            const bool own = j >= c0 && j < c1;
+            if ((which == 0) != own) continue;
+            int slot;
+            if (which == 0) {
+                slot = (int)(j - c0);
+            } else if (colmap) {
+                slot = colmap[j];
+            } else {
+                int lo = 0, hi = sp.nparts - 1;
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if (sp.s[mid] <= j) lo = mid; else hi = mid - 1;
+                }
+                slot = (int)(lo * sp.slot + (j - sp.s[lo]));
+            }
+            col_out[q] = slot;
+            val_out[q] = val[k];
+            ++q;
+        }
+    }
+}
+
 int blocks_for(const spmv_ctx *ctx, int64_t n) {
     return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div<int64_t>(n, 256), (int64_t)ctx->sm_count * 16));
 }
@@ -199,6 +247,52 @@ spmv_status gather_impl(spmv_ctx *ctx, spmv_dtype dt, const void *src, const int
     else k_gather<float><<<blocks_for(ctx, n), 256, 0, s>>>((const float *)src, idx, n, (float *)dst);
     SPMV_LAUNCH_CHECK();
     return SPMV_OK;
+}
+
+template <typename IT, typename V>
+spmv_status split_t(spmv_ctx *ctx, const spmv_csr *A, const int64_t *sp, int nparts, int part, const int32_t *colmap,
+                    int which, cudaStream_t s, int32_t *rp_out, int32_t *col_out, void *val_out, int64_t *nnz_out) {
+    const int64_t r0 = sp[part], rows = sp[part + 1] - sp[part];
+    const IT *rp = (const IT *)A->row_ptr;
+    Scratch cnt(ctx, s), off(ctx, s);
+    SPMV_TRY(cnt.alloc(std::max<int64_t>(rows, 1) * 8));
+    SPMV_TRY(off.alloc((rows + 1) * 8));
+    if (rows) {
+        k_split_count<IT><<<blocks_for(ctx, rows), 256, 0, s>>>(rp, A->col_idx, r0, rows, sp[part], sp[part + 1],
+                                                                which, cnt.as<int64_t>());
+        SPMV_LAUNCH_CHECK();
+    }
+    SPMV_TRY(exclusive_scan_i64(ctx, cnt.as<int64_t>(), off.as<int64_t>(), rows, s));
+    int64_t nnz = 0;
+    SPMV_CUDA_TRY(cudaMemcpyAsync(&nnz, off.as<int64_t>() + rows, 8, cudaMemcpyDeviceToHost, s));
+    SPMV_CUDA_TRY(cudaStreamSynchronize(s));
+    if (nnz > INT32_MAX) { set_error("split block exceeds int32 indices"); return SPMV_ERR_SIZE; }
+    k_i64_to_i32<<<blocks_for(ctx, rows + 1), 256, 0, s>>>(off.as<int64_t>(), rows + 1, rp_out);
+    SPMV_LAUNCH_CHECK();
+    *nnz_out = nnz;
+    if (!col_out || !val_out || nnz == 0 || rows == 0) return SPMV_OK;
+    Splits spl{};
+    int64_t S = 0;
+    for (int k = 0; k <= nparts; ++k) spl.s[k] = sp[k];
+    for (int k = 0; k < nparts; ++k) S = std::max(S, sp[k + 1] - sp[k]);
+    spl.nparts = nparts;
+    spl.slot = S;
+    k_split_fill<IT, V><<<blocks_for(ctx, rows), 256, 0, s>>>(rp, A->col_idx, (const V *)A->vals, r0, rows, sp[part],
+                                                              sp[part + 1], which, spl, colmap, rp_out, col_out,
+                                                              (V *)val_out);
+    SPMV_LAUNCH_CHECK();
+    return SPMV_OK;
+}
+
+spmv_status split_impl(spmv_ctx *ctx, const spmv_csr *A, const int64_t *sp, int nparts, int part,
+                       const int32_t *colmap, int which, cudaStream_t s, int32_t *rp_out, int32_t *col_out,
+                       void *val_out, int64_t *nnz_out) {
+    SPMV_TRY(check_splits(A, sp, nparts));
+    const bool i32 = A->ptr_type == SPMV_I32, f64 = A->dtype == SPMV_F64;
+    if (i32 && f64) return split_t<int, double>(ctx, A, sp, nparts, part, colmap, which, s, rp_out, col_out, val_out, nnz_out);
+    if (i32) return split_t<int, float>(ctx, A, sp, nparts, part, colmap, which, s, rp_out, col_out, val_out, nnz_out);
+    if (f64) return split_t<int64_t, double>(ctx, A, sp, nparts, part, colmap, which, s, rp_out, col_out, val_out, nnz_out);
+    return split_t<int64_t, float>(ctx, A, sp, nparts, part, colmap, which, s, rp_out, col_out, val_out, nnz_out);
 }
 
 spmv_status partition_impl(spmv_ctx *ctx, const spmv_csr *A, int nparts, cudaStream_t s, int64_t *splits) {

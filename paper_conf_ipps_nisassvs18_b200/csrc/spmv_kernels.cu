@@ -493,6 +493,12 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
 // in the tile is written by it (empty rows: beta*y); row r0 may have begun in an
 // earlier tile (its earlier parts arrive as carries); the part of row r1 inside the
 // tile is the tile carry.  The row window is written back coalesced.
+__device__ __forceinline__ int64_t ld_coord(const int64_t *p, uint64_t pol) {
+    int64_t v;
+    asm volatile("ld.global.nc.L2::cache_hint.s64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+    return v;
+}
+
 // N consecutive elements starting at an arbitrary (element-aligned) address: the
 // covering 16-byte vectors, then a shift by the address's offset inside a vector
 template <typename V, int N> struct ShiftLoad;
@@ -546,7 +552,10 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
     unsigned *s_flag = s_flag_all[wid];
     unsigned *s_mark = s_mark_all[wid];
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
-    const int64_t r0 = __ldg(crow + t), k0 = __ldg(cnz + t), r1 = __ldg(crow + t + 1), k1 = __ldg(cnz + t + 1);
+    // tile coordinates: tiny (16 B per tile) and first on the dependency chain -> keep them
+    // L2-resident across runs (evict-last policy)
+    const int64_t r0 = ld_coord(crow + t, px), k0 = ld_coord(cnz + t, px);
+    const int64_t r1 = ld_coord(crow + t + 1, px), k1 = ld_coord(cnz + t + 1, px);
     const int nrows = (int)(r1 - r0), nnzt = (int)(k1 - k0);
     const int j0 = lane * LI;
     const int nv = max(0, min(LI, nnzt - j0));

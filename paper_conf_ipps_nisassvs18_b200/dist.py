@@ -23,7 +23,7 @@ import torch
 import torch.distributed as dist
 
 from .spmv import (CSR, convert, partition, slice_remap, spmv_colmap_pack_index, spmv_gather,
-                   spmv_partition_colmap, spmv_slice_remap_colmap)
+                   spmv_partition_colmap, spmv_slice_remap_colmap, spmv_slice_split)
 
 
 @dataclass
@@ -91,9 +91,13 @@ class DistSpMV:
     partition kernel is deterministic and rank 0's splits are broadcast and checked).
     ``compress=True`` exchanges only the columns some row references:
     slots of S' = max referenced columns per part, packed every step by ``spmv_gather``.
+    ``overlap=True`` splits the shard into its own-column block, run on the rank's x slice
+    while the all-gather is in flight, and its foreign-column block, run (accumulating,
+    beta = 1) once the gather lands.
     """
 
-    def __init__(self, A: CSR, fmt: str = "csr5", group=None, compress: bool = False, **convert_opts):
+    def __init__(self, A: CSR, fmt: str = "csr5", group=None, compress: bool = False, overlap: bool = False,
+                 **convert_opts):
         if A.n_rows != A.n_cols:
             raise ValueError("DistSpMV needs a square matrix (x is owned like y)")
         self.group = group
@@ -118,6 +122,12 @@ class DistSpMV:
             self.pack_idx = None
         self.slot = S
         self.handle = convert(self.shard, fmt, **convert_opts)
+        self.overlap = overlap
+        if overlap:
+            cmap = colmap if compress else None
+            self.own = convert(spmv_slice_split(A, splits, rank, 0), fmt, **convert_opts)
+            self.foreign = convert(spmv_slice_split(A, splits, rank, 1, cmap, S), fmt, **convert_opts)
+            self.x_own = torch.zeros(self.layout.rows, dtype=A.val.dtype, device=dev)
         self.dtype = A.val.dtype
         self.x_slot = torch.zeros(S, dtype=self.dtype, device=dev)
         self.x_gathered = torch.zeros(P * S, dtype=self.dtype, device=dev)
@@ -132,6 +142,8 @@ class DistSpMV:
 
     def set_x(self, x_local: torch.Tensor):
         """Stage this rank's x slice (length rows) into its padded / compressed slot."""
+        if self.overlap:
+            self.x_own.copy_(x_local)
         if self.compress:
             spmv_gather(x_local, self.pack_idx, self.x_slot)
         else:
@@ -139,13 +151,27 @@ class DistSpMV:
 
     def exchange(self):
         """All-gather the x slots (the one collective of a step)."""
-        return all_gather_slots(self.x_gathered, self.x_slot, self.group)
+        torch.cuda.nvtx.range_push("DistSpMV.exchange")
+        try:
+            return all_gather_slots(self.x_gathered, self.x_slot, self.group)
+        finally:
+            torch.cuda.nvtx.range_pop()
 
     def run(self, alpha, beta, y_local: torch.Tensor, x_local: Optional[torch.Tensor] = None):
         """y_local <- alpha*(A x)[r0:r1] + beta*y_local; x_local (optional) replaces the slot."""
         if x_local is not None:
             self.set_x(x_local)
+        if self.overlap and dist.get_backend(self.group) == "nccl":
+            work = dist.all_gather_into_tensor(self.x_gathered, self.x_slot, group=self.group, async_op=True)
+            self.own.run(alpha, self.x_own, beta, y_local)        # overlaps the exchange
+            work.wait()                                           # compute stream waits for the gather
+            self.foreign.run(alpha, self.x_gathered, 1.0, y_local)
+            return y_local
         self.exchange()
+        if self.overlap:
+            self.own.run(alpha, self.x_own, beta, y_local)
+            self.foreign.run(alpha, self.x_gathered, 1.0, y_local)
+            return y_local
         self.handle.run(alpha, self.x_gathered, beta, y_local)
         return y_local
 

@@ -131,6 +131,8 @@ def lib():
             "spmv_colmap_pack_index": (C.c_int, [_P, _P, C.POINTER(C.c_int64), C.c_int, C.c_int, C.c_int64, _P, _P,
                                                  C.POINTER(C.c_int64)]),
             "spmv_gather": (C.c_int, [_P, C.c_int, _P, _P, C.c_int64, _P, _P]),
+            "spmv_slice_split": (C.c_int, [_P, C.POINTER(spmv_csr), C.POINTER(C.c_int64), C.c_int, C.c_int, _P,
+                                           C.c_int, _P, _P, _P, _P, C.POINTER(C.c_int64)]),
             "spmv_status_str": (C.c_char_p, [C.c_int]),
             "spmv_last_error": (C.c_char_p, []),
         }
@@ -358,6 +360,35 @@ def spmv_colmap_pack_index(colmap: torch.Tensor, splits, part: int, slot: int, s
     _check(lib().spmv_colmap_pack_index(ctx.ptr, colmap.data_ptr(), csp, sp.size - 1, int(part), int(slot),
                                         _stream_ptr(stream), idx.data_ptr(), C.byref(cnt)))
     return idx[: cnt.value]
+
+
+def spmv_slice_split(A: CSR, splits, part: int, which: int, colmap: Optional[torch.Tensor] = None,
+                     slot: Optional[int] = None, stream=None) -> CSR:
+    """Own (which=0, columns index the rank's x slice) or foreign (which=1, columns index the
+    gathered x) block of shard `part`."""
+    ctx = context(A.row_ptr.device.index)
+    sp, csp = _splits_c(splits)
+    P = sp.size - 1
+    a = A.as_c()
+    rows = int(sp[part + 1] - sp[part])
+    dev = A.row_ptr.device
+    rp = torch.empty(rows + 1, dtype=torch.int32, device=dev)
+    nnz = C.c_int64()
+    st = _stream_ptr(stream)
+    cm = colmap.data_ptr() if colmap is not None else None
+    _check(lib().spmv_slice_split(ctx.ptr, C.byref(a), csp, P, int(part), cm, int(which), st, rp.data_ptr(), None,
+                                  None, C.byref(nnz)))
+    col = torch.empty(nnz.value, dtype=torch.int32, device=dev)
+    val = torch.empty(nnz.value, dtype=A.val.dtype, device=dev)
+    _check(lib().spmv_slice_split(ctx.ptr, C.byref(a), csp, P, int(part), cm, int(which), st, rp.data_ptr(),
+                                  col.data_ptr() if nnz.value else None, val.data_ptr() if nnz.value else None,
+                                  C.byref(nnz)))
+    if which == 0:
+        n_cols = rows
+    else:
+        S = slot if slot is not None else int(np.max(np.diff(sp)))
+        n_cols = P * S
+    return CSR(rp, col, val, (rows, n_cols))
 
 
 def spmv_gather(src: torch.Tensor, idx: torch.Tensor, dst: torch.Tensor, stream=None):

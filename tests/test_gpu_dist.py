@@ -140,3 +140,47 @@ def test_distspmv_nccl_world1_compressed(sp):
         assert oracle.check_tolerance(yl.cpu().numpy(), ref, bound, 1e-12)[0]
     finally:
         dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("compress", [False, True])
+@pytest.mark.parametrize("P", [2, 4])
+def test_own_foreign_split_bit_exact(sp, P, compress):
+    from paper_conf_ipps_nisassvs18_b200.spmv import spmv_partition_colmap, spmv_slice_split
+    A = matgen.rmat(13, seed=51)
+    dA = sp.CSR.from_host(A)
+    splits = sp.partition(dA, P)
+    if compress:
+        cm, S = spmv_partition_colmap(dA, splits)
+        cm_o, _ = oracle.partition_colmap(A, splits)
+    else:
+        cm, S, cm_o = None, None, None
+    for k in range(P):
+        for which in (0, 1):
+            blk = spmv_slice_split(dA, splits, k, which, cm, S)
+            rp, col, val = oracle.slice_split(A, splits, k, which, cm_o)
+            assert np.array_equal(blk.row_ptr.cpu().numpy().astype(np.int64), rp)
+            assert np.array_equal(blk.col.cpu().numpy(), col)
+            assert np.array_equal(blk.val.cpu().numpy(), val)
+
+
+@pytest.mark.parametrize("compress", [False, True])
+def test_distspmv_nccl_world1_overlap(sp, compress):
+    import torch.distributed as dist
+    from paper_conf_ipps_nisassvs18_b200.dist import DistSpMV
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK="0", WORLD_SIZE="1")
+    dist.init_process_group("nccl", device_id=torch.device("cuda", 0))
+    try:
+        A = matgen.rmat(12, seed=45)
+        x = matgen.vector(A.n_cols, 45, 1)
+        y = matgen.vector(A.n_rows, 45, 2)
+        ref, bound = oracle.spmv_csr(A, x, 2.0, 0.5, y, with_bound=True)
+        D = DistSpMV(sp.CSR.from_host(A), "csr5", compress=compress, overlap=True)
+        yl = torch.from_numpy(y.copy()).cuda()
+        D.run(2.0, 0.5, yl, x_local=torch.from_numpy(x).cuda())
+        assert oracle.check_tolerance(yl.cpu().numpy(), ref, bound, 1e-12)[0]
+    finally:
+        dist.destroy_process_group()

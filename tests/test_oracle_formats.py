@@ -379,3 +379,38 @@ def test_compressed_exchange_reassembles_spmv(P):
         rp, col, val = oracle.slice_remap_colmap(A, s, k, cm)
         shard = matgen.HostCSR(rp, col, val, int(s[k + 1] - s[k]), P * S)
         assert np.array_equal(oracle.spmv_csr(shard, xg, 0.5, 2.0, y[s[k]:s[k + 1]]), full[s[k]:s[k + 1]])
+
+
+@pytest.mark.parametrize("compress", [False, True])
+@pytest.mark.parametrize("P", [1, 2, 4])
+def test_own_foreign_split_reassembles(P, compress):
+    """SURVEY §8(e) 2: own block (x slice) + foreign block (gathered x) = the shard's product;
+    the two blocks partition the shard's nonzeros."""
+    A = matgen.rmat(10, seed=29)
+    x = matgen.vector(A.n_cols, 29, 1)
+    y = matgen.vector(A.n_rows, 29, 2)
+    s = oracle.partition(A, P)
+    ref, bound = oracle.spmv_csr(A, x, 1.5, -0.5, y, with_bound=True)
+    if compress:
+        cm, S = oracle.partition_colmap(A, s)
+    else:
+        cm, S = None, oracle.partition_slot(s)
+    xg = np.zeros(P * S)
+    for k in range(P):
+        if compress:
+            js = np.nonzero(cm[s[k]:s[k + 1]] >= 0)[0] + s[k]
+            xg[k * S:k * S + js.size] = x[js]
+        else:
+            xg[k * S:k * S + s[k + 1] - s[k]] = x[s[k]:s[k + 1]]
+    for k in range(P):
+        r0, r1 = int(s[k]), int(s[k + 1])
+        rpo, co, vo = oracle.slice_split(A, s, k, 0, cm)
+        rpf, cf, vf = oracle.slice_split(A, s, k, 1, cm)
+        assert co.size + cf.size == A.row_ptr[r1] - A.row_ptr[r0]
+        assert np.all((co >= 0) & (co < r1 - r0))
+        own = matgen.HostCSR(rpo, co, vo, r1 - r0, r1 - r0)
+        foreign = matgen.HostCSR(rpf, cf, vf, r1 - r0, P * S)
+        part = oracle.spmv_csr(own, x[r0:r1], 1.5, -0.5, y[r0:r1])
+        part = oracle.spmv_csr(foreign, xg, 1.5, 1.0, part)
+        ok, ratio, _ = oracle.check_tolerance(part, ref[r0:r1], bound[r0:r1], 1e-13)
+        assert ok, ratio
