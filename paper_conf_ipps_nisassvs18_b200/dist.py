@@ -123,10 +123,9 @@ class DistSpMV:
         self.slot = S
         self.handle = convert(self.shard, fmt, **convert_opts)
         self.overlap = overlap
+        self._A, self._colmap = A, (colmap if compress else None)
         if overlap:
-            cmap = colmap if compress else None
-            self.own = convert(spmv_slice_split(A, splits, rank, 0), fmt, **convert_opts)
-            self.foreign = convert(spmv_slice_split(A, splits, rank, 1, cmap, S), fmt, **convert_opts)
+            self.own, self.foreign = self.split_handles(fmt, **convert_opts)
             self.x_own = torch.zeros(self.layout.rows, dtype=A.val.dtype, device=dev)
         self.dtype = A.val.dtype
         self.x_slot = torch.zeros(S, dtype=self.dtype, device=dev)
@@ -135,6 +134,21 @@ class DistSpMV:
     @property
     def rows(self) -> int:
         return self.layout.rows
+
+    def split_handles(self, fmt: str, **convert_opts):
+        """(own-column block, foreign-column block) of this rank's shard in format `fmt`."""
+        lay = self.layout
+        own = convert(spmv_slice_split(self._A, lay.splits, lay.rank, 0), fmt, **convert_opts)
+        foreign = convert(spmv_slice_split(self._A, lay.splits, lay.rank, 1, self._colmap, self.slot), fmt,
+                          **convert_opts)
+        return own, foreign
+
+    def exchange_async(self):
+        """Start the all-gather; returns the work handle (NCCL) or None (completed)."""
+        if dist.get_backend(self.group) == "nccl":
+            return dist.all_gather_into_tensor(self.x_gathered, self.x_slot, group=self.group, async_op=True)
+        self.exchange()
+        return None
 
     def exchange_bytes(self) -> int:
         """Bytes each rank receives per step."""
