@@ -538,22 +538,16 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
         int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
     constexpr int TI = 32 * LI;                           // merge-path items per warp tile
     static_assert(LI == 4 || LI == 8, "lane chunk of 4 or 8 items");
-    __shared__ double s_sum_all[kT / 32][TI];             // row sums (local row index)
+    __shared__ double s_sum_all[kT / 32][TI];             // segment sum, keyed by its start position
     __shared__ int s_end_all[kT / 32][TI];                // local end of local row i
-    __shared__ unsigned short s_rowat_all[kT / 32][TI];   // local row starting at a position
-    __shared__ unsigned s_flag_all[kT / 32][TI / 32];
-    __shared__ unsigned s_mark_all[kT / 32][TI / 32];
+    __shared__ unsigned s_flag_all[kT / 32][TI / 32];     // segment-start bitmap over the tile's nonzeros
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     if (t >= n_tiles) return;
     double *s_sum = s_sum_all[wid];
     int *s_end = s_end_all[wid];
-    unsigned short *s_rowat = s_rowat_all[wid];
     unsigned *s_flag = s_flag_all[wid];
-    unsigned *s_mark = s_mark_all[wid];
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
-    // tile coordinates: tiny (16 B per tile) and first on the dependency chain -> keep them
-    // L2-resident across runs (evict-last policy)
     const int64_t r0 = ld_coord(crow + t, px), k0 = ld_coord(cnz + t, px);
     const int64_t r1 = ld_coord(crow + t + 1, px), k1 = ld_coord(cnz + t + 1, px);
     const int nrows = (int)(r1 - r0), nnzt = (int)(k1 - k0);
@@ -573,71 +567,67 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
     }
     for (int i = lane; i < nrows; i += 32) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
     const bool r0_inside = (int64_t)__ldg(rp + r0) == k0;   // A7: rp[r0] <= k0 always
-    if (lane < TI / 32) { s_flag[lane] = 0u; s_mark[lane] = 0u; }
+    if (lane < TI / 32) s_flag[lane] = 0u;
     double p[LI];
 #pragma unroll
-    for (int s = 0; s < LI; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
+    for (int e = 0; e < LI; ++e) p[e] = e < nv ? (double)v[e] * (double)ld_x(x + c[e], px) : 0.0;
     __syncwarp();
     // segment starts: local row i (1 <= i <= nrows) starts at s_end[i-1]; row 0 at 0 if r0_inside
     for (int i = lane; i <= nrows; i += 32) {
         const int st = i == 0 ? 0 : s_end[i - 1];
         const int en = i < nrows ? s_end[i] : nnzt;         // open row r1 runs past the tile
-        if ((i > 0 || r0_inside) && st < nnzt && en > st) {
-            atomicOr(&s_flag[st >> 5], 1u << (st & 31));
-            s_rowat[st] = (unsigned short)i;
-        }
+        if ((i > 0 || r0_inside) && st < nnzt && en > st) atomicOr(&s_flag[st >> 5], 1u << (st & 31));
     }
+    // where the open row r1 starts inside the tile (its segment is the tile carry), else -1
+    const int open_start = nrows > 0 ? (s_end[nrows - 1] < nnzt ? s_end[nrows - 1] : -1) : (r0_inside && nnzt > 0 ? 0 : -1);
     __syncwarp();
     const unsigned fl = nv > 0 ? ((s_flag[j0 >> 5] >> (j0 & 31)) & ((1u << LI) - 1u)) : 0u;
-    auto put = [&](int li, double sum) {
-        s_sum[li] = sum;
-        atomicOr(&s_mark[li >> 5], 1u << (li & 31));
-    };
     double acc = 0.0, head = 0.0;
     int kseg = 0, cur = -1;
 #pragma unroll
-    for (int s = 0; s < LI; ++s) {
-        if ((fl >> s) & 1u) {
+    for (int e = 0; e < LI; ++e) {
+        if ((fl >> e) & 1u) {
             if (kseg == 0) head = acc;
-            else put(cur, acc);                           // closed inside the lane (cur < nrows)
+            else s_sum[cur] = acc;                        // segment closed inside the lane
             ++kseg;
-            cur = s_rowat[j0 + s];
+            cur = j0 + e;
             acc = 0.0;
         }
-        acc += p[s];
+        acc += p[e];
     }
     if (kseg == 0) head = acc;
     double Rnext;
     const double R = seg_suffix(head, kseg > 0 || nv == 0, &Rnext);
-    const double lead = __shfl_sync(0xffffffffu, R, 0);  // nonzeros before the tile's first segment
+    const double lead = __shfl_sync(0xffffffffu, R, 0);  // nonzeros before the tile's first segment start
     double cv = 0.0;
     int cset = 0;
     if (kseg > 0) {
         const double tot = acc + Rnext;
-        if (cur < nrows) put(cur, tot);
+        if (cur != open_start) s_sum[cur] = tot;
         else { cv = tot; cset = 1; }                      // row r1 started in this tile
     }
-    if (lane == 0 && !r0_inside && nnzt > 0) {
-        if (nrows > 0) put(0, lead);                      // row r0 ends here
-        else { cv = lead; cset = 1; }                     // the tile is the middle of row r0 == r1
-    }
+    if (lane == 0 && !r0_inside && nnzt > 0 && nrows == 0) { cv = lead; cset = 1; }   // middle of row r0 == r1
     const unsigned who = __ballot_sync(0xffffffffu, cset);
     if (lane == 0 && who == 0) { carry_row[t] = -1; carry_val[t] = 0.0; }
     if (cset) { carry_row[t] = r1; carry_val[t] = cv; }
     __syncwarp();
+    // every row ending in the tile: its segment sum (row 0 begun earlier: the lead run)
+    auto row_sum = [&](int i) -> double {
+        const int st = i == 0 ? 0 : s_end[i - 1];
+        if (i == 0 && !r0_inside) return lead;
+        return s_end[i] > st ? s_sum[st] : 0.0;
+    };
 #pragma unroll
     for (int q = 0; q < kOutQ; ++q) {
         const int i = lane + 32 * q;
         if (i < nrows) {
-            const bool marked = (s_mark[i >> 5] >> (i & 31)) & 1u;
-            double o = marked ? alpha * s_sum[i] : 0.0;
+            double o = alpha * row_sum(i);
             if (!B0) o = fma(beta, yv[q], o);
             y[r0 + i] = (V)o;
         }
     }
     for (int i = kOutWin + lane; i < nrows; i += 32) {        // rows beyond the prefetched window
-        const bool marked = (s_mark[i >> 5] >> (i & 31)) & 1u;
-        double o = marked ? alpha * s_sum[i] : 0.0;
+        double o = alpha * row_sum(i);
         if (!B0) o = fma(beta, (double)y[r0 + i], o);
         y[r0 + i] = (V)o;
     }
