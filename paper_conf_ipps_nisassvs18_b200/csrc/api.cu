@@ -254,7 +254,8 @@ spmv_status spmv_info(const spmv_handle *h, spmv_handle_info *o) {
     size_t dev = 0, fmt_bytes = 0;
     for (int i = 0; i < kMaxArrays; ++i) {
         if (h->arr[i].owned) dev += h->arr[i].bytes;
-        fmt_bytes += h->arr[i].bytes;
+        // the merge kernel derives the nonzero coordinate as d - row (A7): kept for export, not read
+        if (i != SPMV_ARR_MERGE_COORD_NZ) fmt_bytes += h->arr[i].bytes;
     }
     dev += h->carry_row.bytes + h->carry_val.bytes;
     o->device_bytes = dev;
