@@ -137,7 +137,8 @@ typedef struct {
     size_t max_bytes;      /* ELL/HYB guard (0 = min(1/2 free memory, max(8x the CSR bytes,
                               64 MiB)))                                                    */
     int alias_input;       /* 1 = COO/CSR handles reference the caller's col/vals (caller
-                              keeps them alive and unchanged); MERGE/CSR5/ELL/HYB copy     */
+                              keeps them alive and unchanged); MERGE/CSR5/ELL/HYB copy,
+                              and COO copies unless both arrays are 32-byte aligned        */
     int index64;           /* 1 = int64 row pointers/offsets inside the handle even when
                               nnz <= INT32_MAX (exercises the > 2^31-nonzero path, A17)   */
 } spmv_convert_opts;

@@ -107,6 +107,28 @@ __device__ __forceinline__ double4a ld_hint(const double4a *p, uint64_t pol) {
     r.hi = ld_hint(reinterpret_cast<const double2 *>(p) + 1, pol);
     return r;
 }
+// 256-bit (32-byte aligned) streaming loads: one instruction covers a whole sector per
+// lane, so a lane's 8-element chunk is requested from L2 once (two 16-byte loads of one
+// sector would be two requests -- with L1::no_allocate the second goes to L2 again)
+__device__ __forceinline__ void ld256(const int *p, int (&v)[8], uint64_t pol) {
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+                 : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+                 : "l"(p), "l"(pol));
+}
+__device__ __forceinline__ void ld256(const float *p, float (&v)[8], uint64_t pol) {
+    int w[8];
+    ld256(reinterpret_cast<const int *>(p), w, pol);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = __int_as_float(w[i]);
+}
+__device__ __forceinline__ void ld256(const double *p, double (&v)[4], uint64_t pol) {
+    long long w[4];
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.b64 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=l"(w[0]), "=l"(w[1]), "=l"(w[2]), "=l"(w[3]) : "l"(p), "l"(pol));
+#pragma unroll
+    for (int i = 0; i < 4; ++i) v[i] = __longlong_as_double(w[i]);
+}
+
 // x gathers: read-only path, keep in L1 (neighbouring gathers hit), L2 evict-last
 __device__ __forceinline__ float ld_x(const float *p, uint64_t pol) {
     float v;
@@ -116,6 +138,11 @@ __device__ __forceinline__ float ld_x(const float *p, uint64_t pol) {
 __device__ __forceinline__ double ld_x(const double *p, uint64_t pol) {
     double v;
     asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ int ld_x(const int *p, uint64_t pol) {
+    int v;
+    asm volatile("ld.global.nc.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
 

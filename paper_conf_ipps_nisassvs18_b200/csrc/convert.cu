@@ -7,6 +7,8 @@
 #include <algorithm>
 #include <climits>
 
+#include <cstdint>
+
 #include "internal.h"
 #include "kernels.h"
 #include "scan.h"
@@ -286,7 +288,9 @@ spmv_status convert_t(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, const s
         break;
     }
     case SPMV_COO: {
-        SPMV_TRY(copy_colval(o->alias_input != 0));
+        // the COO kernel reads 32-byte lane chunks: alias only 32-byte aligned arrays
+        const bool al32 = (((uintptr_t)col | (uintptr_t)val) & 31) == 0;
+        SPMV_TRY(copy_colval(o->alias_input != 0 && al32));
         SPMV_TRY(arr_alloc(h, SPMV_ARR_COO_ROW, nnz * 4, s));
         if (nnz) {
             k_walk<IT><<<walk_grid, kT, 0, s>>>(rp, n, nnz, OpCoo{(int *)h->arr[SPMV_ARR_COO_ROW].p});

@@ -19,9 +19,6 @@
 #include "internal.h"
 #include "kernels.h"
 
-#ifndef SPMV_MERGE_SHFL
-#define SPMV_MERGE_SHFL 1
-#endif
 
 namespace spmv {
 
@@ -65,8 +62,8 @@ __global__ void k_scale(V *y, int64_t n, double beta) {
 // folded every kFold steps, A13) -- the paper's warp-per-row kernel for long rows.
 template <int W> struct VecCfg { static constexpr int U = W <= 8 ? 32 / (32 / W) : (W == 16 ? 4 : 2); };
 
-template <typename V, typename IT, int W, bool B0>
-__global__ void __launch_bounds__(kT, 3)
+template <typename V, typename IT, int W, bool B0, int MB>
+__global__ void __launch_bounds__(kT, MB)
 k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
              const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta) {
     constexpr int G = 32 / W;
@@ -341,32 +338,21 @@ constexpr int kOutQ = kOutWin / 32;
 // rows between the tile's rows and up to the next tile's first row get beta*y.  The
 // tile's row window is staged in shared memory and written back coalesced.
 // ACCUM (HYB's COO part): y += alpha*s for rows present, nothing else.
+// 8 consecutive elements from a 32-byte aligned address, 256-bit loads
 template <typename V> struct VecLoad8;
 template <> struct VecLoad8<double> {
     static __device__ __forceinline__ void load(const double *p, double (&v)[8], uint64_t pol) {
+        double a[4], b[4];
+        ld256(p, a, pol);
+        ld256(p + 4, b, pol);
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            double2 w = ld_hint(reinterpret_cast<const double2 *>(p) + q, pol);
-            v[2 * q] = w.x; v[2 * q + 1] = w.y;
-        }
+        for (int q = 0; q < 4; ++q) { v[q] = a[q]; v[4 + q] = b[q]; }
     }
 };
 template <> struct VecLoad8<float> {
-    static __device__ __forceinline__ void load(const float *p, float (&v)[8], uint64_t pol) {
-#pragma unroll
-        for (int q = 0; q < 2; ++q) {
-            float4 w = ld_hint(reinterpret_cast<const float4 *>(p) + q, pol);
-            v[4 * q] = w.x; v[4 * q + 1] = w.y; v[4 * q + 2] = w.z; v[4 * q + 3] = w.w;
-        }
-    }
+    static __device__ __forceinline__ void load(const float *p, float (&v)[8], uint64_t pol) { ld256(p, v, pol); }
 };
-__device__ __forceinline__ void load_int8(const int *p, int (&v)[8], uint64_t pol) {
-#pragma unroll
-    for (int q = 0; q < 2; ++q) {
-        int4 w = ld_hint(reinterpret_cast<const int4 *>(p) + q, pol);
-        v[4 * q] = w.x; v[4 * q + 1] = w.y; v[4 * q + 2] = w.z; v[4 * q + 3] = w.w;
-    }
-}
+__device__ __forceinline__ void load_int8(const int *p, int (&v)[8], uint64_t pol) { ld256(p, v, pol); }
 
 template <typename V, bool ACCUM, bool B0>
 __global__ void __launch_bounds__(kT, kMinBlocks)
@@ -536,46 +522,49 @@ template <int N> struct ShiftLoad<int, N> {
 };
 
 // N consecutive elements starting at offset m (warp-uniform, < E) past the lane's
-// aligned chunk b = base + N*lane: the lane loads only its own aligned vectors (E
-// elements each) and takes the m elements that spill into the next chunk from lane+1
-// by shuffle; lane 31 loads that next vector itself.  Every A sector is requested
-// once (the shifted loads re-request each chunk boundary from L2).
-template <typename T, typename VT, int E, int N>
+// 32-byte aligned chunk b = base + N*lane: the lane loads only its own chunk (256-bit
+// loads of E elements, so each sector is requested once) and takes the m elements that
+// spill into the next chunk from lane+1 by shuffle; lane 31 loads that vector itself.
+// The shift by m is a log shifter (warp-uniform branches).
+template <typename T> struct Vec256 { static constexpr int E = 32 / sizeof(T); };
+template <typename T, int N>
 __device__ __forceinline__ void shfl_load(const T *b, int m, bool load, bool extra, T (&v)[N], uint64_t pol) {
-    static_assert(N % E == 0, "whole vectors per lane");
-    T w[N], nb[E - 1];
+    constexpr int E = Vec256<T>::E;
+    static_assert(N % E == 0, "whole 32-byte vectors per lane");
+    T w[N + E - 1];
 #pragma unroll
     for (int q = 0; q < N / E; ++q) {
-        VT t;
-        if (load) t = ld_hint(reinterpret_cast<const VT *>(b) + q, pol);
-        else std::memset(&t, 0, sizeof t);
-        const T *tp = reinterpret_cast<const T *>(&t);
+        T t[E];
+        if (load) ld256(b + q * E, t, pol);
+        else {
 #pragma unroll
-        for (int e = 0; e < E; ++e) w[q * E + e] = tp[e];
+            for (int e = 0; e < E; ++e) t[e] = T(0);
+        }
+#pragma unroll
+        for (int e = 0; e < E; ++e) w[q * E + e] = t[e];
     }
-    VT xt;
-    if (extra) xt = ld_hint(reinterpret_cast<const VT *>(b) + N / E, pol);
-    else std::memset(&xt, 0, sizeof xt);
-    const T *xp = reinterpret_cast<const T *>(&xt);
+    T xt[E];
+    if (extra) ld256(b + N, xt, pol);
+    else {
+#pragma unroll
+        for (int e = 0; e < E; ++e) xt[e] = T(0);
+    }
     const bool last = (threadIdx.x & 31) == 31;
 #pragma unroll
     for (int e = 0; e < E - 1; ++e) {
         const T s = __shfl_down_sync(0xffffffffu, w[e], 1);
-        nb[e] = last ? xp[e] : s;
+        w[N + e] = last ? xt[e] : s;
     }
 #pragma unroll
-    for (int i = 0; i < N; ++i) {
-        T r = w[i];
+    for (int bit = E / 2; bit > 0; bit >>= 1) {
+        if (m & bit) {
 #pragma unroll
-        for (int d = 1; d < E; ++d)
-            if (m == d) r = i + d < N ? w[i + d] : nb[i + d - N];
-        v[i] = r;
+            for (int i = 0; i + bit < N + E - 1; ++i) w[i] = w[i + bit];
+        }
     }
+#pragma unroll
+    for (int i = 0; i < N; ++i) v[i] = w[i];
 }
-template <typename V> struct VecOf;
-template <> struct VecOf<double> { using T = double2; static constexpr int E = 2; };
-template <> struct VecOf<float> { using T = float4; static constexpr int E = 4; };
-template <> struct VecOf<int> { using T = int4; static constexpr int E = 4; };
 
 template <typename V, typename IT, bool B0, int LI>
 __device__ __forceinline__ void
@@ -590,21 +579,17 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
     const int nv = max(0, min(LI, nnzt - j0));
     int c[LI];
     V v[LI];
-#if SPMV_MERGE_SHFL
-    {
-        // aligned chunks: col by 4, val by VecOf<V>::E elements; both alignments warp-uniform
-        const int mc = (int)(k0 & 3), mv = (int)(k0 & (VecOf<V>::E - 1));
+    if constexpr (LI == 8) {
+        // 32-byte aligned chunks: col by 8, val by Vec256<V>::E elements; offsets warp-uniform
+        constexpr int EV = Vec256<V>::E;
+        const int mc = (int)(k0 & 7), mv = (int)(k0 & (EV - 1));
         const bool lc = j0 < mc + nnzt, lv = j0 < mv + nnzt;
-        shfl_load<int, int4, 4, LI>(col + (k0 - mc) + j0, mc, lc, lane == 31 && 32 * LI < mc + nnzt, c, pa);
-        shfl_load<V, typename VecOf<V>::T, VecOf<V>::E, LI>(val + (k0 - mv) + j0, mv, lv,
-                                                            lane == 31 && 32 * LI < mv + nnzt, v, pa);
-    }
-#else
-    if (nv > 0) {
+        shfl_load<int, LI>(col + (k0 - mc) + j0, mc, lc, lane == 31 && 32 * LI < mc + nnzt, c, pa);
+        shfl_load<V, LI>(val + (k0 - mv) + j0, mv, lv, lane == 31 && 32 * LI < mv + nnzt, v, pa);
+    } else if (nv > 0) {                                  // 4-item lane chunks: shifted 16-byte loads
         ShiftLoad<int, LI>::load(col + k0 + j0, c, pa);
         ShiftLoad<V, LI>::load(val + k0 + j0, v, pa);
     }
-#endif
     double yv[kOutQ];
 #pragma unroll
     for (int q = 0; q < kOutQ; ++q) {
@@ -970,7 +955,9 @@ spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col
     // 16 CTAs (4096 threads) per SM of grid-stride warps
     const int64_t threads = ceil_div<int64_t>(n, 32 / w) * 32;
     const int g = grid_stride_blocks(h->ctx, threads, 16);
-#define SPMV_VEC(WW) k_csr_vector<V, IT, WW, B0><<<g, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta)
+    // W <= 8: 4 CTAs/SM (64 registers; LAP4096 0.442 -> 0.384 ms); wider groups keep
+    // 3 CTAs/SM (80 registers; R-MAT 24 at W = 16: 4 CTAs/SM 11 % slower)
+#define SPMV_VEC(WW) k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3)><<<g, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta)
     switch (w) {
     case 1: case 2: SPMV_VEC(2); break;
     case 4: SPMV_VEC(4); break;

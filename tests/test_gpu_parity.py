@@ -447,3 +447,25 @@ def test_index64_path(sp, name, fmt, dtype):
         e = oracle.csr5_encode(A, val_bytes=8 if dtype == torch.float64 else 4)
         assert np.array_equal(h.export("csr5_tile_desc"), e["tile_desc"])
         assert np.array_equal(h.export("row_ptr"), A.row_ptr)
+
+
+@pytest.mark.parametrize("offset", [0, 1, 3])
+@pytest.mark.parametrize("fmt", ("coo", "csr", "merge", "csr5"))
+def test_alias_input_any_alignment(sp, fmt, offset):
+    """alias_input with col/val slices starting `offset` elements into their buffers: a
+    handle that references them must not assume vector alignment (COO copies unless both
+    are 32-byte aligned, include/spmv.h), and results stay within tolerance."""
+    A = case("rmat15", "f64")
+    dA = to_dev(sp, A, torch.float64)
+    cb = torch.zeros(A.nnz + 8, dtype=torch.int32, device="cuda")
+    vb = torch.zeros(A.nnz + 8, dtype=torch.float64, device="cuda")
+    cb[offset: offset + A.nnz] = dA.col
+    vb[offset: offset + A.nnz] = dA.val
+    dS = sp.CSR(dA.row_ptr, cb[offset: offset + A.nnz], vb[offset: offset + A.nnz], (A.n_rows, A.n_cols))
+    x = matgen.vector(A.n_cols, 78, 1)
+    y0 = matgen.vector(A.n_rows, 78, 2)
+    ref, bound = oracle.spmv_csr(A, x, 1.5, -0.5, y0, with_bound=True)
+    h, out = run_format(sp, A, dS, fmt, torch.float64, 1.5, -0.5, x, y0, alias_input=1)
+    ok, ratio, nbad = oracle.check_tolerance(out, ref, bound, TOL[torch.float64])
+    assert ok, f"{fmt} offset {offset}: {nbad} bad rows, max ratio {ratio}"
+    h.destroy()
