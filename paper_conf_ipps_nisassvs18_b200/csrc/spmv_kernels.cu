@@ -475,12 +475,15 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
 // rows into equal sized sub-problems".  Warp w owns merge-path diagonals
 // [w*T, (w+1)*T) of (row ends) x (nonzeros), T = kMergeItems: rows [r0, r1) end in
 // the tile and nonzeros [k0, k1) are consumed by it (coordinates precomputed at
-// conversion, A7).  Lane l takes the tile's nonzeros [8l, 8l+8): every lane chunk has
-// the same misalignment (k0 mod 4), so the lane loads the covering 16-byte vectors
-// and shifts them by that warp-uniform amount -- products stay in registers with
-// all x gathers in flight.  The tile's row ends (coalesced, shared) mark segment
-// starts in a 256-bit shared bitmap; each lane then reduces its chunk like a CSR5
-// lane (in-lane segments + flag-segmented suffix sum over lanes).  Every row ending
+// conversion, A7; only the row coordinate is read, the nonzero one is d - row).
+// Lane l takes the 32-byte aligned chunk of 8 nonzeros [base + 8l, base + 8l + 8),
+// base = k0 rounded down to 8 elements, with 256-bit loads (each sector requested
+// once); positions outside the tile are masked, and the <= 7 positions past lane 31's
+// chunk (tiles with < 8 row ends) are a short extra loop of lane 31.  Products stay in
+// registers with all x gathers in flight.  The tile's row ends (coalesced, shared)
+// mark segment starts in a shared bitmap over chunk positions; each lane then reduces
+// its chunk like a CSR5 lane (in-lane segments + flag-segmented suffix sum).
+// Persistent warps prefetch the next tile's row coordinates.  Every row ending
 // in the tile is written by it (empty rows: beta*y); row r0 may have begun in an
 // earlier tile (its earlier parts arrive as carries); the part of row r1 inside the
 // tile is the tile carry.  The row window is written back coalesced.
@@ -521,51 +524,6 @@ template <int N> struct ShiftLoad<int, N> {
     static __device__ __forceinline__ void load(const int *p, int (&v)[N], uint64_t pol) { shift_load4<int, int4, N>(p, v, pol); }
 };
 
-// N consecutive elements starting at offset m (warp-uniform, < E) past the lane's
-// 32-byte aligned chunk b = base + N*lane: the lane loads only its own chunk (256-bit
-// loads of E elements, so each sector is requested once) and takes the m elements that
-// spill into the next chunk from lane+1 by shuffle; lane 31 loads that vector itself.
-// The shift by m is a log shifter (warp-uniform branches).
-template <typename T> struct Vec256 { static constexpr int E = 32 / sizeof(T); };
-template <typename T, int N>
-__device__ __forceinline__ void shfl_load(const T *b, int m, bool load, bool extra, T (&v)[N], uint64_t pol) {
-    constexpr int E = Vec256<T>::E;
-    static_assert(N % E == 0, "whole 32-byte vectors per lane");
-    T w[N + E - 1];
-#pragma unroll
-    for (int q = 0; q < N / E; ++q) {
-        T t[E];
-        if (load) ld256(b + q * E, t, pol);
-        else {
-#pragma unroll
-            for (int e = 0; e < E; ++e) t[e] = T(0);
-        }
-#pragma unroll
-        for (int e = 0; e < E; ++e) w[q * E + e] = t[e];
-    }
-    T xt[E];
-    if (extra) ld256(b + N, xt, pol);
-    else {
-#pragma unroll
-        for (int e = 0; e < E; ++e) xt[e] = T(0);
-    }
-    const bool last = (threadIdx.x & 31) == 31;
-#pragma unroll
-    for (int e = 0; e < E - 1; ++e) {
-        const T s = __shfl_down_sync(0xffffffffu, w[e], 1);
-        w[N + e] = last ? xt[e] : s;
-    }
-#pragma unroll
-    for (int bit = E / 2; bit > 0; bit >>= 1) {
-        if (m & bit) {
-#pragma unroll
-            for (int i = 0; i + bit < N + E - 1; ++i) w[i] = w[i + bit];
-        }
-    }
-#pragma unroll
-    for (int i = 0; i < N; ++i) v[i] = w[i];
-}
-
 template <typename V, typename IT, bool B0, int LI>
 __device__ __forceinline__ void
 merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val, int64_t t,
@@ -575,18 +533,22 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
     constexpr int TI = 32 * LI;
     const int lane = threadIdx.x & 31;
     const int nrows = (int)(r1 - r0), nnzt = (int)(k1 - k0);
-    const int j0 = lane * LI;
-    const int nv = max(0, min(LI, nnzt - j0));
+    // LI = 8: lane l owns the 32-byte aligned chunk [base + 8l, base + 8l + 8), base =
+    // k0 - off: tile positions [8l - off, 8l - off + 8), those outside [0, nnzt) masked,
+    // so no shifting; positions [256 - off, nnzt) (a tile with < 8 row ends) are one
+    // more chunk, taken by lane 31.  LI = 4: shifted 16-byte loads (off = 0).
+    const int off = LI == 8 ? (int)(k0 & 7) : 0;
+    const int64_t base = k0 - off;
+    const int j0 = lane * LI - off;                        // tile position of the lane's first element
+    const bool any = j0 < nnzt;                            // the lane holds a tile element
     int c[LI];
     V v[LI];
     if constexpr (LI == 8) {
-        // 32-byte aligned chunks: col by 8, val by Vec256<V>::E elements; offsets warp-uniform
-        constexpr int EV = Vec256<V>::E;
-        const int mc = (int)(k0 & 7), mv = (int)(k0 & (EV - 1));
-        const bool lc = j0 < mc + nnzt, lv = j0 < mv + nnzt;
-        shfl_load<int, LI>(col + (k0 - mc) + j0, mc, lc, lane == 31 && 32 * LI < mc + nnzt, c, pa);
-        shfl_load<V, LI>(val + (k0 - mv) + j0, mv, lv, lane == 31 && 32 * LI < mv + nnzt, v, pa);
-    } else if (nv > 0) {                                  // 4-item lane chunks: shifted 16-byte loads
+        if (any) {
+            ld256(col + base + lane * LI, c, pa);
+            VecLoad8<V>::load(val + base + lane * LI, v, pa);
+        }
+    } else if (any) {
         ShiftLoad<int, LI>::load(col + k0 + j0, c, pa);
         ShiftLoad<V, LI>::load(val + k0 + j0, v, pa);
     }
@@ -598,21 +560,26 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
     }
     for (int i = lane; i < nrows; i += 32) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
     const bool r0_inside = (int64_t)__ldg(rp + r0) == k0;   // A7: rp[r0] <= k0 always
-    if (lane < TI / 32) s_flag[lane] = 0u;
+    if (lane <= TI / 32) s_flag[lane] = 0u;
     double p[LI];
 #pragma unroll
-    for (int e = 0; e < LI; ++e) p[e] = e < nv ? (double)v[e] * (double)ld_x(x + c[e], px) : 0.0;
+    for (int e = 0; e < LI; ++e)
+        p[e] = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)v[e] * (double)ld_x(x + c[e], px) : 0.0;
     __syncwarp();
-    // segment starts: local row i (1 <= i <= nrows) starts at s_end[i-1]; row 0 at 0 if r0_inside
+    // segment starts: local row i (1 <= i <= nrows) starts at s_end[i-1]; row 0 at 0 if
+    // r0_inside.  The bitmap is indexed by chunk position (tile position + off).
     for (int i = lane; i <= nrows; i += 32) {
         const int st = i == 0 ? 0 : s_end[i - 1];
         const int en = i < nrows ? s_end[i] : nnzt;         // open row r1 runs past the tile
-        if ((i > 0 || r0_inside) && st < nnzt && en > st) atomicOr(&s_flag[st >> 5], 1u << (st & 31));
+        if ((i > 0 || r0_inside) && st < nnzt && en > st) {
+            const int q = st + off;
+            atomicOr(&s_flag[q >> 5], 1u << (q & 31));
+        }
     }
     // where the open row r1 starts inside the tile (its segment is the tile carry), else -1
     const int open_start = nrows > 0 ? (s_end[nrows - 1] < nnzt ? s_end[nrows - 1] : -1) : (r0_inside && nnzt > 0 ? 0 : -1);
     __syncwarp();
-    const unsigned fl = nv > 0 ? ((s_flag[j0 >> 5] >> (j0 & 31)) & ((1u << LI) - 1u)) : 0u;
+    const unsigned fl = any ? ((s_flag[(lane * LI) >> 5] >> ((lane * LI) & 31)) & ((1u << LI) - 1u)) : 0u;
     double acc = 0.0, head = 0.0;
     int kseg = 0, cur = -1;
 #pragma unroll
@@ -626,7 +593,25 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
         }
         acc += p[e];
     }
+    if constexpr (LI == 8) {
+        if (lane == 31 && j0 + LI < nnzt) {               // overflow chunk (rare: long rows)
+            const unsigned fl2 = s_flag[TI / 32] & 0xFFu;
+#pragma unroll 1
+            for (int pos = j0 + LI; pos < nnzt; ++pos) {
+                const int e = pos - (j0 + LI);
+                if ((fl2 >> e) & 1u) {
+                    if (kseg == 0) head = acc;
+                    else s_sum[cur] = acc;
+                    ++kseg;
+                    cur = pos;
+                    acc = 0.0;
+                }
+                acc += (double)ld_hint(val + k0 + pos, pa) * (double)ld_x(x + ld_hint(col + k0 + pos, pa), px);
+            }
+        }
+    }
     if (kseg == 0) head = acc;
+    const int nv = any ? 1 : 0;
     double Rnext;
     const double R = seg_suffix(head, kseg > 0 || nv == 0, &Rnext);
     const double lead = __shfl_sync(0xffffffffu, R, 0);  // nonzeros before the tile's first segment start
@@ -680,7 +665,7 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
     constexpr int TI = 32 * LI;
     __shared__ double s_sum_all[kT / 32][TI];             // segment sum, keyed by its start position
     __shared__ int s_end_all[kT / 32][TI];                // local end of local row i
-    __shared__ unsigned s_flag_all[kT / 32][TI / 32];     // segment-start bitmap over the tile's nonzeros
+    __shared__ unsigned s_flag_all[kT / 32][TI / 32 + 1]; // segment-start bitmap over the lane chunks
     const int wid = threadIdx.x >> 5;
     const int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     if (t >= n_tiles) return;
@@ -702,7 +687,7 @@ k_merge_persist(const IT *__restrict__ rp, const int *__restrict__ col, const V 
     constexpr int TI = 32 * LI;
     __shared__ double s_sum_all[kT / 32][TI];
     __shared__ int s_end_all[kT / 32][TI];
-    __shared__ unsigned s_flag_all[kT / 32][TI / 32];
+    __shared__ unsigned s_flag_all[kT / 32][TI / 32 + 1];
     const int wid = threadIdx.x >> 5;
     const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
     int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
