@@ -29,6 +29,21 @@ def short(name):
     return n
 
 
+SPMV_KERNELS = ("k_coo", "k_ell", "k_csr_vector", "k_merge", "k_merge_persist", "k_csr5")
+B0_ARG = {"k_coo": 2, "k_ell": 1, "k_csr_vector": 3, "k_merge": 2, "k_merge_persist": 2, "k_csr5": 3}
+
+
+def targs(name):
+    return [a.strip() for a in name.split("<", 1)[1].rsplit(">", 1)[0].split(",")] if "<" in name else []
+
+
+def is_beta0(name):
+    """True for the beta == 0 instantiation of an SpMV kernel (not launched by a bench step)."""
+    base, a = name.split("<")[0], targs(name)
+    i = B0_ARG.get(base)
+    return i is not None and i < len(a) and a[i] in ("1", "true")
+
+
 def launches(path, out):
     rows = list(csv.reader(open(path)))
     i = [k for k, r in enumerate(rows) if "Kernel Name" in r][0]
@@ -54,9 +69,9 @@ def launches(path, out):
             share = f"{100 * s / tot:.1f}%" if k in spmv and tot else "-"
             f.write(f"| `{k}` | {len(v)} | {s / len(v):.1f} | {s:.1f} | {share} |\n")
         # share of one timed step: the step's SpMV launches (beta != 0 variants, fix-ups)
-        step = {k: sum(v) / len(v) * (2 if k.startswith("k_ell<") and "1>" not in k else 1)
-                for k, v in agg.items()
-                if k.split("<")[0] in ("k_coo", "k_ell", "k_csr_vector", "k_merge", "k_csr5") and not k.endswith("1>")}
+        # (ELL's kernel runs twice per step when HYB is all-ELL, as on LAP4096: K_h = K)
+        step = {k: sum(v) / len(v) * (2 if k.startswith("k_ell<") else 1)
+                for k, v in agg.items() if k.split("<")[0] in SPMV_KERNELS and not is_beta0(k)}
         fix = agg.get("k_fixup<double>") or agg.get("k_fixup<float>")
         if fix:
             step["k_fixup (x launches per step)"] = sum(fix) / len(fix) * 3
@@ -111,10 +126,10 @@ def full(rep, out, traffic=None, formats=("coo", "ell", "csr", "hyb", "merge", "
         lines.append(f"| `{name}` | " + " | ".join(cells) + f" | {top} |")
         base = name.split("<")[0]
         seen[base] += 1
-        targs = name.split("<")[1] if "<" in name else ""
-        fmt = {"k_merge": "merge", "k_csr5": "csr5"}.get(base)
+        ta = targs(name)
+        fmt = {"k_merge": "merge", "k_merge_persist": "merge", "k_csr5": "csr5"}.get(base)
         if base == "k_coo":
-            fmt = "hyb" if targs.split(",")[1].strip() in ("1", "true") else "coo"
+            fmt = "hyb" if ta[1] in ("1", "true") else "coo"
         elif base == "k_ell":
             fmt = "ell" if ("ell" in formats and seen[base] == 1) else "hyb"
         elif base == "k_csr_vector" and seen[base] == 1 and "csr" in formats:
