@@ -112,15 +112,31 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
         double s[U];
 #pragma unroll
         for (int u = 0; u < U; ++u) s[u] = c0[u] >= 0 ? (double)v0[u] * (double)ld_x(x + c0[u], px) : 0.0;
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-#pragma unroll
-            for (int o = W / 2; o > 0; o >>= 1) s[u] += __shfl_xor_sync(0xffffffffu, s[u], o);
-        }
         // the group's U results: lane sub == u of group g writes row u*G + g
         double mine = 0.0;
+        {
+            // lane bits >= U do not index rows: plain butterflies over them; then a
+            // transpose reduction over the low bits -- at offset o a lane keeps the half
+            // of its partial sums selected by (sub & o) and adds the other half received
+            // from lane sub ^ o, so lane sub ends with row (sub mod U)'s sum (U - 1
+            // shuffles instead of a butterfly per row, U * log2(U))
 #pragma unroll
-        for (int u = 0; u < U; ++u) mine = (sub == u) ? s[u] : mine;
+            for (int o = W / 2; o >= U; o >>= 1) {
+#pragma unroll
+                for (int u = 0; u < U; ++u) s[u] += __shfl_xor_sync(0xffffffffu, s[u], o);
+            }
+#pragma unroll
+            for (int o = U / 2; o > 0; o >>= 1) {
+                const bool hi = (sub & o) != 0;
+#pragma unroll
+                for (int j = 0; j < o; ++j) {
+                    const double send = hi ? s[j] : s[j + o];
+                    const double keep = hi ? s[j + o] : s[j];
+                    s[j] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+                }
+            }
+            mine = s[0];
+        }
         // rows longer than W: the remainder is processed by the WHOLE warp, one row at a
         // time (the paper's warp-per-row vector kernel), 8 loads per lane in
         // flight, accumulators folded every kFold steps (A13); lane i holds row i's range
