@@ -419,7 +419,14 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
         const int i = lane + 32 * q;
         yv[q] = ((ACCUM || !B0) && i < L) ? (double)y[Wlo + i] : 0.0;
     }
-    if (lane < kOutWin / 32) s_mark[lane] = 0u;
+    // window rows without a segment (empty rows) keep s = 0: y = alpha*0 + beta*y, as the
+    // definition (c1) reads; only ACCUM (rows present only) needs the row marks
+    if (ACCUM) {
+        if (lane < kOutWin / 32) s_mark[lane] = 0u;
+    } else {
+#pragma unroll
+        for (int q = 0; q < kOutQ; ++q) s_acc[lane + 32 * q] = 0.0;
+    }
     double p[8];
 #pragma unroll
     for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
@@ -429,7 +436,7 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
         const int64_t li = rr - Wlo;
         if (li >= 0 && li < kOutWin) {
             s_acc[li] = sum;
-            atomicOr(&s_mark[li >> 5], 1u << (li & 31));
+            if (ACCUM) atomicOr(&s_mark[li >> 5], 1u << (li & 31));
         } else if (ACCUM) {
             y[rr] = (V)((double)y[rr] + alpha * sum);
         } else {
@@ -474,12 +481,11 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
     for (int q = 0; q < kOutQ; ++q) {
         const int i = lane + 32 * q;
         if (i < L) {
-            const bool marked = (s_mark[i >> 5] >> (i & 31)) & 1u;
             if (ACCUM) {
-                if (marked) y[Wlo + i] = (V)(yv[q] + alpha * s_acc[i]);
+                if ((s_mark[i >> 5] >> (i & 31)) & 1u) y[Wlo + i] = (V)(yv[q] + alpha * s_acc[i]);
             } else {
-                double o = marked ? alpha * s_acc[i] : 0.0;
-                if (!B0) o = marked ? fma(beta, yv[q], o) : beta * yv[q];
+                double o = alpha * s_acc[i];
+                if (!B0) o = fma(beta, yv[q], o);
                 y[Wlo + i] = (V)o;
             }
         }
@@ -497,7 +503,7 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
 // once); positions outside the tile are masked, and the <= 7 positions past lane 31's
 // chunk (tiles with < 8 row ends) are a short extra loop of lane 31.  Products stay in
 // registers with all x gathers in flight.  The tile's row ends (coalesced, shared)
-// mark segment starts in a shared bitmap over chunk positions; each lane then reduces
+// mark segment starts as shared byte flags over chunk positions; each lane then reduces
 // its chunk like a CSR5 lane (in-lane segments + flag-segmented suffix sum).
 // Persistent warps prefetch the next tile's row coordinates.  Every row ending
 // in the tile is written by it (empty rows: beta*y); row r0 may have begun in an
@@ -545,7 +551,7 @@ __device__ __forceinline__ void
 merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val, int64_t t,
            int64_t r0, int64_t r1, int64_t k0, int64_t k1, const V *__restrict__ x, V *__restrict__ y,
            double alpha, double beta, int64_t *__restrict__ carry_row, double *__restrict__ carry_val,
-           double *s_sum, int *s_end, unsigned *s_flag, uint64_t pa, uint64_t px) {
+           double *s_sum, int *s_end, uint2 *s_flag, uint64_t pa, uint64_t px) {
     constexpr int TI = 32 * LI;
     const int lane = threadIdx.x & 31;
     const int nrows = (int)(r1 - r0), nnzt = (int)(k1 - k0);
@@ -576,7 +582,9 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
     }
     for (int i = lane; i < nrows; i += 32) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
     const bool r0_inside = (int64_t)__ldg(rp + r0) == k0;   // A7: rp[r0] <= k0 always
-    if (lane <= TI / 32) s_flag[lane] = 0u;
+    // segment-start flags, one byte per chunk position (plain stores, no atomics)
+    unsigned char *s_fb = reinterpret_cast<unsigned char *>(s_flag);
+    for (int i = lane; i < TI / 8 + 1; i += 32) s_flag[i] = make_uint2(0u, 0u);
     double p[LI];
 #pragma unroll
     for (int e = 0; e < LI; ++e)
@@ -588,14 +596,24 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
         const int st = i == 0 ? 0 : s_end[i - 1];
         const int en = i < nrows ? s_end[i] : nnzt;         // open row r1 runs past the tile
         if ((i > 0 || r0_inside) && st < nnzt && en > st) {
-            const int q = st + off;
-            atomicOr(&s_flag[q >> 5], 1u << (q & 31));
+            s_fb[st + off] = 1;
         }
     }
     // where the open row r1 starts inside the tile (its segment is the tile carry), else -1
     const int open_start = nrows > 0 ? (s_end[nrows - 1] < nnzt ? s_end[nrows - 1] : -1) : (r0_inside && nnzt > 0 ? 0 : -1);
     __syncwarp();
-    const unsigned fl = any ? ((s_flag[(lane * LI) >> 5] >> ((lane * LI) & 31)) & ((1u << LI) - 1u)) : 0u;
+    // bytes (0/1) of the lane's chunk -> bit mask: (b & 0x01010101) * 0x01020408 gathers the
+    // four low bits into the top byte without carries
+    auto pack4 = [](unsigned w) -> unsigned { return ((w & 0x01010101u) * 0x01020408u) >> 24; };
+    unsigned fl = 0u;
+    if (any) {
+        if constexpr (LI == 8) {
+            const uint2 w = s_flag[lane];
+            fl = pack4(w.x) | (pack4(w.y) << 4);
+        } else {
+            fl = pack4(reinterpret_cast<const unsigned *>(s_flag)[lane]);
+        }
+    }
     double acc = 0.0, head = 0.0;
     int kseg = 0, cur = -1;
 #pragma unroll
@@ -611,7 +629,8 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
     }
     if constexpr (LI == 8) {
         if (lane == 31 && j0 + LI < nnzt) {               // overflow chunk (rare: long rows)
-            const unsigned fl2 = s_flag[TI / 32] & 0xFFu;
+            const uint2 w2 = s_flag[TI / 8];
+            const unsigned fl2 = pack4(w2.x) | (pack4(w2.y) << 4);
 #pragma unroll 1
             for (int pos = j0 + LI; pos < nnzt; ++pos) {
                 const int e = pos - (j0 + LI);
@@ -681,7 +700,7 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
     constexpr int TI = 32 * LI;
     __shared__ double s_sum_all[kT / 32][TI];             // segment sum, keyed by its start position
     __shared__ int s_end_all[kT / 32][TI];                // local end of local row i
-    __shared__ unsigned s_flag_all[kT / 32][TI / 32 + 1]; // segment-start bitmap over the lane chunks
+    __shared__ uint2 s_flag_all[kT / 32][TI / 8 + 1];     // segment-start byte flags over the lane chunks
     const int wid = threadIdx.x >> 5;
     const int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     if (t >= n_tiles) return;
@@ -703,7 +722,7 @@ k_merge_persist(const IT *__restrict__ rp, const int *__restrict__ col, const V 
     constexpr int TI = 32 * LI;
     __shared__ double s_sum_all[kT / 32][TI];
     __shared__ int s_end_all[kT / 32][TI];
-    __shared__ unsigned s_flag_all[kT / 32][TI / 32 + 1];
+    __shared__ uint2 s_flag_all[kT / 32][TI / 8 + 1];
     const int wid = threadIdx.x >> 5;
     const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
     int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -772,7 +791,6 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
     constexpr int64_t W = 32 * SIGMA;
     constexpr int kQ = kCsr5Win / 32;
     __shared__ double s_acc[kT / 32][kCsr5Win];
-    __shared__ unsigned s_mark[kT / 32][kCsr5Win / 32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     if (t > n_tiles) return;
@@ -814,7 +832,9 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
         const int i = lane + 32 * q;
         yv[q] = (!B0 && i < L) ? (double)y[lo + i] : 0.0;
     }
-    if (lane < kCsr5Win / 32) s_mark[wid][lane] = 0u;
+    // empty window rows keep s = 0: y = alpha*0 + beta*y, as the definition (c1) reads
+#pragma unroll
+    for (int q = 0; q < kQ; ++q) s_acc[wid][lane + 32 * q] = 0.0;
     double p[SIGMA];
 #pragma unroll
     for (int s = 0; s < SIGMA; ++s) p[s] = (double)v[s] * (double)ld_x(x + c[s], px);
@@ -828,7 +848,6 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
         const int64_t li = r - lo;
         if (li < kCsr5Win) {
             s_acc[wid][li] = sum;
-            atomicOr(&s_mark[wid][li >> 5], 1u << (li & 31));
         } else {
             y_write<V, B0>(y, r, sum, alpha, beta);
         }
@@ -868,14 +887,13 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
         carry_val[t] = lead ? R : 0.0;
     }
     __syncwarp();
-    // write the window: segment rows alpha*s + beta*y, empty rows beta*y
+    // write the window: alpha*s + beta*y (s = 0 for empty rows)
 #pragma unroll
     for (int q = 0; q < kQ; ++q) {
         const int i = lane + 32 * q;
         if (i < L) {
-            const bool marked = (s_mark[wid][i >> 5] >> (i & 31)) & 1u;
-            double o = marked ? alpha * s_acc[wid][i] : 0.0;
-            if (!B0) o = marked ? fma(beta, yv[q], o) : beta * yv[q];
+            double o = alpha * s_acc[wid][i];
+            if (!B0) o = fma(beta, yv[q], o);
             y[lo + i] = (V)o;
         }
     }
