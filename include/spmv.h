@@ -35,7 +35,7 @@ extern "C" {
 #pragma GCC visibility push(default)
 #endif
 
-#define SPMV_ABI_VERSION 1
+#define SPMV_ABI_VERSION 2
 
 typedef enum {
     SPMV_OK = 0,
@@ -141,6 +141,9 @@ typedef struct {
                               and COO copies unless both arrays are 32-byte aligned        */
     int index64;           /* 1 = int64 row pointers/offsets inside the handle even when
                               nnz <= INT32_MAX (exercises the > 2^31-nonzero path, A17)   */
+    int64_t csr_chunk;     /* CSR long-row split (A25): rows longer than 2*csr_chunk are cut
+                              into csr_chunk-nonzero chunks, each reduced by its own warp and
+                              added by the fix-up; 0 = default 512, < 0 = never split     */
 } spmv_convert_opts;
 
 /* Fill `opts` with the defaults (all rules as above). */
@@ -183,6 +186,7 @@ typedef struct {
     int64_t csr5_sigma, csr5_tiles, csr5_map_len;
     int64_t merge_items, merge_tiles;
     int64_t vector_width;
+    int64_t csr_chunks;             /* CSR long-row chunks (A25); 0 = none */
     size_t device_bytes;            /* bytes owned by the handle */
     size_t bytes_per_run;           /* algorithmic bytes of one run with beta != 0
                                        (format's own storage + x + y read + y write),
@@ -208,7 +212,9 @@ typedef enum {
     SPMV_ARR_CSR5_ROW_LO = 11,      /* int64 [tiles+1] */
     SPMV_ARR_CSR5_TILE_DESC = 12,   /* uint32 [tiles*32] */
     SPMV_ARR_CSR5_MAP_OFF = 13,     /* int64 [tiles] (-1 = no empty row in range) */
-    SPMV_ARR_CSR5_SEG_MAP = 14      /* int64 [map_len] */
+    SPMV_ARR_CSR5_SEG_MAP = 14,     /* int64 [map_len] */
+    SPMV_ARR_CSR_CHUNK_ROW = 15,    /* CSR: int64 [chunks], row of each long-row chunk (A25) */
+    SPMV_ARR_CSR_CHUNK_LO = 16      /* CSR: int64 [chunks], first nonzero of each chunk      */
 } spmv_array_id;
 
 /* Copy array `id` of the handle to host memory (blocking on `stream`).

@@ -77,6 +77,7 @@ def lib():
             "ora_hyb_coo_nnz": (_i64, [_i64, _p, _i64]),
             "ora_csr2hyb": (C.c_int, [_i64, _p, _p, _p, _i64, _i64, _p, _p, _p, _p, _p]),
             "ora_merge_ntiles": (_i64, [_i64, _i64, _i64]),
+            "ora_csr_chunks": (_i64, [_i64, _p, _i64, _p, _p]),
             "ora_merge_coords": (C.c_int, [_i64, _p, _i64, _p, _p]),
             "ora_csr5_sigma": (_i64, [_i64, _i64]),
             "ora_csr5_map_len": (_i64, [_i64, _p, _i64]),
@@ -221,6 +222,16 @@ def merge_coords(A, T):
     rc = lib().ora_merge_coords(A.n_rows, _ptr(A.row_ptr), int(T), _ptr(cr), _ptr(cn))
     assert rc == 0
     return cr, cn
+
+
+def csr_chunks(A, C):
+    """CSR long-row chunks (A25): (chunk_row, chunk_lo) int64 arrays."""
+    A = CSR.of(A)
+    m = int(lib().ora_csr_chunks(A.n_rows, _ptr(A.row_ptr), int(C), None, None))
+    assert m >= 0
+    cr, cl = _buf(max(m, 1), np.int64), _buf(max(m, 1), np.int64)
+    lib().ora_csr_chunks(A.n_rows, _ptr(A.row_ptr), int(C), _ptr(cr), _ptr(cl))
+    return cr[:m], cl[:m]
 
 
 def csr5_sigma(A):

@@ -196,6 +196,23 @@ int ora_csr2hyb(int64_t n_rows, const int64_t *row_ptr, const int32_t *col,
 /* Merge-based CSR: "logically partitions the work ... into equal
  * sized sub-problems".  Work items = n_rows row ends + nnz nonzeros; tile t takes
  * diagonals [t*T, (t+1)*T). */
+int64_t ora_csr_chunks(int64_t n_rows, const int64_t *row_ptr, int64_t C,
+                       int64_t *chunk_row, int64_t *chunk_lo)
+{
+    if (C <= 0 || n_rows < 0) return -1;
+    int64_t k = 0;
+    for (int64_t r = 0; r < n_rows; ++r) {
+        int64_t len = row_ptr[r + 1] - row_ptr[r];
+        if (len <= 2 * C) continue;
+        for (int64_t start = row_ptr[r]; start < row_ptr[r + 1]; start += C) {
+            if (chunk_row) chunk_row[k] = r;
+            if (chunk_lo) chunk_lo[k] = start;
+            ++k;
+        }
+    }
+    return k;
+}
+
 int64_t ora_merge_ntiles(int64_t n_rows, int64_t nnz, int64_t T)
 {
     if (T <= 0) return -1;

@@ -76,6 +76,13 @@ int64_t ora_merge_ntiles(int64_t n_rows, int64_t nnz, int64_t T);
 int ora_merge_coords(int64_t n_rows, const int64_t *row_ptr, int64_t T,
                      int64_t *coord_row, int64_t *coord_nz);
 
+/* CSR long-row chunks (A25): a row with len > 2*C is reduced as
+ * ceil(len/C) chunks of C nonzeros (the last one shorter), chunk j of row r starting at
+ * row_ptr[r] + j*C; chunks listed by ascending row, then j.  Returns the number of
+ * chunks (negative on bad input); chunk_row/chunk_lo (nullable) receive them. */
+int64_t ora_csr_chunks(int64_t n_rows, const int64_t *row_ptr, int64_t C,
+                       int64_t *chunk_row, int64_t *chunk_lo);
+
 /* CSR5 (encoding of SURVEY A6, restated in DESIGN.md §4.6).
  * omega = 32 lanes, sigma from ora_csr5_sigma.  n_tiles = floor(nnz/(omega*sigma)).
  * Outputs (caller-sized):

@@ -251,6 +251,7 @@ spmv_status spmv_info(const spmv_handle *h, spmv_handle_info *o) {
     o->merge_items = h->merge_T;
     o->merge_tiles = h->merge_tiles;
     o->vector_width = h->vec_w;
+    o->csr_chunks = h->csr_chunks;
     size_t dev = 0, fmt_bytes = 0;
     for (int i = 0; i < kMaxArrays; ++i) {
         if (h->arr[i].owned) dev += h->arr[i].bytes;
@@ -278,7 +279,8 @@ spmv_status spmv_export(const spmv_handle *h, spmv_array_id id, void *dst, size_
         bool present = false;
         switch (h->fmt) {
         case SPMV_COO: present = id == SPMV_ARR_COO_ROW || id == SPMV_ARR_COL || id == SPMV_ARR_VAL; break;
-        case SPMV_CSR: case SPMV_CSR_SCALAR: present = id <= SPMV_ARR_VAL; break;
+        case SPMV_CSR: present = id <= SPMV_ARR_VAL || id == SPMV_ARR_CSR_CHUNK_ROW || id == SPMV_ARR_CSR_CHUNK_LO; break;
+        case SPMV_CSR_SCALAR: present = id <= SPMV_ARR_VAL; break;
         case SPMV_ELL: present = id == SPMV_ARR_ELL_COL || id == SPMV_ARR_ELL_VAL; break;
         case SPMV_HYB: present = id == SPMV_ARR_ELL_COL || id == SPMV_ARR_ELL_VAL || id == SPMV_ARR_COO_ROW ||
                                  id == SPMV_ARR_HYB_COO_COL || id == SPMV_ARR_HYB_COO_VAL; break;

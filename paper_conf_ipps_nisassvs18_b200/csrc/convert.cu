@@ -89,6 +89,24 @@ __global__ void k_hyb_overflow(const IT *rp, int64_t n, int64_t kh, int64_t *cnt
     }
 }
 
+// CSR long-row split (A25): rows longer than 2C become ceil(len/C) chunks of C nonzeros
+template <typename IT>
+__global__ void k_chunk_count(const IT *rp, int64_t n, int64_t C, int64_t *cnt) {
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t len = (int64_t)rp[r + 1] - (int64_t)rp[r];
+        cnt[r] = len > 2 * C ? (len + C - 1) / C : 0;
+    }
+}
+template <typename IT>
+__global__ void k_chunk_fill(const IT *rp, int64_t n, int64_t C, const int64_t *off, int64_t *crow, int64_t *clo) {
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t a = rp[r], len = (int64_t)rp[r + 1] - a;
+        if (len <= 2 * C) continue;
+        const int64_t o = off[r], m = (len + C - 1) / C;
+        for (int64_t j = 0; j < m; ++j) { crow[o + j] = r; clo[o + j] = a + j * C; }
+    }
+}
+
 // merge-path tile coordinates at diagonals min(t*T, n+nnz) (A7)
 template <typename IT>
 __global__ void k_merge_coords(const IT *rp, int64_t n, int64_t nnz, int64_t T, int64_t tiles,
@@ -285,6 +303,32 @@ spmv_status convert_t(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, const s
             while (w < mu && w < 32) w <<= 1;
         }
         h->vec_w = fmt == SPMV_CSR_SCALAR ? 1 : w;
+        if (fmt == SPMV_CSR && o->csr_chunk >= 0) {
+            // long rows (> 2C nonzeros) as C-nonzero chunks, one warp each, added by the fix-up (A25)
+            const int64_t C = o->csr_chunk > 0 ? o->csr_chunk : kCsrChunk;
+            h->csr_chunk = C;
+            Scratch cnt(ctx, s), off(ctx, s);
+            SPMV_TRY(cnt.alloc(std::max<int64_t>(n, 1) * 8));
+            SPMV_TRY(off.alloc((n + 1) * 8));
+            if (n) {
+                k_chunk_count<IT><<<grid_cap(ctx, n), kT, 0, s>>>(rp, n, C, cnt.as<int64_t>());
+                SPMV_LAUNCH_CHECK();
+            }
+            SPMV_TRY(exclusive_scan_i64(ctx, cnt.as<int64_t>(), off.as<int64_t>(), n, s));
+            int64_t nch = 0;
+            SPMV_CUDA_TRY(cudaMemcpyAsync(&nch, off.as<int64_t>() + n, 8, cudaMemcpyDeviceToHost, s));
+            SPMV_CUDA_TRY(cudaStreamSynchronize(s));
+            h->csr_chunks = nch;
+            SPMV_TRY(arr_alloc(h, SPMV_ARR_CSR_CHUNK_ROW, nch * 8, s));
+            SPMV_TRY(arr_alloc(h, SPMV_ARR_CSR_CHUNK_LO, nch * 8, s));
+            if (nch) {
+                k_chunk_fill<IT><<<grid_cap(ctx, n), kT, 0, s>>>(rp, n, C, off.as<int64_t>(),
+                                                                  (int64_t *)h->arr[SPMV_ARR_CSR_CHUNK_ROW].p,
+                                                                  (int64_t *)h->arr[SPMV_ARR_CSR_CHUNK_LO].p);
+                SPMV_LAUNCH_CHECK();
+            }
+            h->n_carry = nch;
+        }
         break;
     }
     case SPMV_COO: {

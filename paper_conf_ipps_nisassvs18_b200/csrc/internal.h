@@ -12,7 +12,7 @@ struct spmv_ctx {
 
 namespace spmv {
 
-constexpr int kMaxArrays = 15;
+constexpr int kMaxArrays = 17;
 
 struct DevArray {
     void *p = nullptr;
@@ -74,6 +74,7 @@ struct spmv_handle {
     int64_t csr5_tail_row = 0;     // first row starting in the CSR5 tail (host copy of row_lo[n_tiles])
     int64_t merge_T = 0, merge_tiles = 0;
     int64_t vec_w = 0;
+    int64_t csr_chunk = 0, csr_chunks = 0;   // CSR long-row split (A25): chunk length, chunk count
     // per-run scratch: carries (row, value) of CTAs/tiles for the fix-up pass
     spmv::DevArray carry_row, carry_val;
     int64_t n_carry = 0;

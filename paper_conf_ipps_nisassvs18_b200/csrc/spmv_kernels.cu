@@ -62,10 +62,10 @@ __global__ void k_scale(V *y, int64_t n, double beta) {
 // folded every kFold steps, A13) -- the paper's warp-per-row kernel for long rows.
 template <int W> struct VecCfg { static constexpr int U = W <= 8 ? 32 / (32 / W) : (W == 16 ? 4 : 2); };
 
-template <typename V, typename IT, int W, bool B0, int MB>
+template <typename V, typename IT, int W, bool B0, int MB, bool CHUNKED>
 __global__ void __launch_bounds__(kT, MB)
 k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
-             const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta) {
+             const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta, int64_t long_len) {
     constexpr int G = 32 / W;
     constexpr int U = (VecCfg<W>::U * G > 32) ? 32 / G : VecCfg<W>::U;
     constexpr int R = G * U;                      // rows per warp iteration (<= 32)
@@ -96,6 +96,7 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
             const IT nx = __shfl_sync(0xffffffffu, rp_lo, (i + 1) & 31);
             b[u] = i + 1 < R ? nx : rp_hi;
             if (base + i >= n) { a[u] = 0; b[u] = 0; }
+            if (CHUNKED && (int64_t)b[u] - (int64_t)a[u] > long_len) b[u] = a[u];   // chunked long row (A25): beta*y here
         }
         // the y value this lane will write (writer lane sub == u of group g: row u*G + g)
         const int64_t my_row = base + (int64_t)sub * G + g;
@@ -144,7 +145,8 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
             const IT my_a = rp_lo;
             const IT my_b = __shfl_sync(0xffffffffu, rp_lo, (lane + 1) & 31);
             const IT my_e = lane + 1 < R ? my_b : rp_hi;
-            unsigned more = __ballot_sync(0xffffffffu, lane < R && base + lane < n && (int64_t)my_e - (int64_t)my_a > W);
+            const int64_t my_len = (int64_t)my_e - (int64_t)my_a;
+            unsigned more = __ballot_sync(0xffffffffu, lane < R && base + lane < n && my_len > W && (!CHUNKED || my_len <= long_len));
             while (more) {
                 const int i = __ffs(more) - 1;
                 more &= more - 1;
@@ -180,6 +182,46 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
             if (!B0) o = fma(beta, yv, o);
             y[my_row] = (V)o;
         }
+    }
+}
+
+// ------------------------------------------------------------------ CSR long-row chunks (A25)
+// One warp per C-nonzero chunk of a long row (8 loads per lane in flight, blocked
+// summation, A13); the chunk sum is the carry (row, value) that the fix-up adds in
+// chunk order.  The row-batch kernel wrote beta*y for these rows.
+template <typename V, typename IT>
+__global__ void __launch_bounds__(kT)
+k_csr_chunks(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
+             const int64_t *__restrict__ crow, const int64_t *__restrict__ clo, int64_t nch, int64_t C,
+             const V *__restrict__ x, int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t pa = policy_evict_first(), px = policy_evict_last();
+    for (int64_t c = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; c < nch;
+         c += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        const int64_t r = __ldg(crow + c), lo = __ldg(clo + c);
+        const int64_t re = (int64_t)__ldg(rp + r + 1);
+        const int64_t hi = lo + C < re ? lo + C : re;
+        double tot = 0.0, acc[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc[q] = 0.0;
+        int it = 0;
+        int64_t k = lo + lane;
+        for (; k + 7 * 32 < hi; k += 8 * 32) {
+            int d[8];
+            V w[8];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
+#pragma unroll
+            for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(x + d[q], px);
+            if (++it == kFold) {
+#pragma unroll
+                for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
+                it = 0;
+            }
+        }
+        for (; k < hi; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
+        const double part = warp_sum(tot + (((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]))));
+        if (lane == 0) { carry_row[c] = r; carry_val[c] = part; }
     }
 }
 
@@ -969,14 +1011,19 @@ spmv_status launch_ell(spmv_handle *h, const V *x, V *y, double alpha, double be
 
 template <typename V, typename IT, bool B0>
 spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col, const V *val, const V *x, V *y,
-                              int64_t n, int w, double alpha, double beta, cudaStream_t s) {
+                              int64_t n, int w, double alpha, double beta, cudaStream_t s,
+                              int64_t long_len = INT64_MAX) {
     if (n == 0) return SPMV_OK;
     // 16 CTAs (4096 threads) per SM of grid-stride warps
     const int64_t threads = ceil_div<int64_t>(n, 32 / w) * 32;
     const int g = grid_stride_blocks(h->ctx, threads, 16);
     // W <= 8: 4 CTAs/SM (64 registers; LAP4096 0.442 -> 0.384 ms); wider groups keep
     // 3 CTAs/SM (80 registers; R-MAT 24 at W = 16: 4 CTAs/SM 11 % slower)
-#define SPMV_VEC(WW) k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3)><<<g, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta)
+#define SPMV_VEC(WW)                                                                                           \
+    if (long_len == INT64_MAX)                                                                                 \
+        k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false><<<g, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len); \
+    else                                                                                                       \
+        k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true><<<g, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len)
     switch (w) {
     case 1: case 2: SPMV_VEC(2); break;
     case 4: SPMV_VEC(4); break;
@@ -1000,7 +1047,18 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
     double *cval = (double *)h->carry_val.p;
     switch (h->fmt) {
     case SPMV_CSR:
-        return launch_csr_vector<V, IT, B0>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s);
+    {
+        if (h->csr_chunks == 0) return launch_csr_vector<V, IT, B0>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s);
+        SPMV_TRY((launch_csr_vector<V, IT, B0>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s,
+                                               2 * h->csr_chunk)));
+        const int64_t warps = h->csr_chunks;
+        const unsigned gc = (unsigned)std::min<int64_t>(ceil_div<int64_t>(warps, kT / 32), (int64_t)h->ctx->sm_count * 16);
+        k_csr_chunks<V, IT><<<gc, kT, 0, s>>>(rp, col, val, (const int64_t *)h->arr[SPMV_ARR_CSR_CHUNK_ROW].p,
+                                              (const int64_t *)h->arr[SPMV_ARR_CSR_CHUNK_LO].p, h->csr_chunks,
+                                              h->csr_chunk, x, crow, cval);
+        SPMV_LAUNCH_CHECK();
+        return launch_fixup<V>(h, y, alpha, s);
+    }
     case SPMV_CSR_SCALAR:
         if (n == 0) return SPMV_OK;
         k_csr_scalar<V, IT, B0><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta);
@@ -1092,7 +1150,8 @@ spmv_status run_impl(spmv_handle *h, double alpha, double beta, const void *x, v
 int run_launch_count(const spmv_handle *h, bool alpha0) {
     if (alpha0) return h->n_rows ? 1 : 0;
     switch (h->fmt) {
-    case SPMV_CSR: case SPMV_CSR_SCALAR: case SPMV_ELL: return h->n_rows ? 1 : 0;
+    case SPMV_CSR: return h->n_rows ? 1 + (h->csr_chunks ? 2 : 0) : 0;
+    case SPMV_CSR_SCALAR: case SPMV_ELL: return h->n_rows ? 1 : 0;
     case SPMV_HYB: return (h->n_rows ? 1 : 0) + (h->hyb_coo_nnz ? 2 : 0);
     case SPMV_COO: return h->nnz ? 2 : (h->n_rows ? 1 : 0);
     case SPMV_MERGE: return h->merge_tiles ? 2 : 0;

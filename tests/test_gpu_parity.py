@@ -469,3 +469,46 @@ def test_alias_input_any_alignment(sp, fmt, offset):
     ok, ratio, nbad = oracle.check_tolerance(out, ref, bound, TOL[torch.float64])
     assert ok, f"{fmt} offset {offset}: {nbad} bad rows, max ratio {ratio}"
     h.destroy()
+
+
+# ------------------------------------------------------------------ CSR long-row chunks (A25)
+
+@pytest.mark.parametrize("chunk", [1, 7, 32, 300])
+@pytest.mark.parametrize("name", ["dense_row_1x5000", "long_row", "rmat15", "empty_runs", "tile_bounds", "u2048"])
+def test_csr_long_row_chunks(sp, name, chunk):
+    """CSR with rows longer than 2*chunk split into chunks (one warp each, carries + fix-up):
+    chunk arrays equal the oracle's bit for bit, results within tolerance for every
+    (alpha, beta), bit-exact in the integer regime."""
+    A = case(name, "f64")
+    dA = to_dev(sp, A, torch.float64)
+    h = sp.convert(dA, "csr", csr_chunk=chunk)
+    cr, cl = oracle.csr_chunks(A, chunk)
+    assert h.info()["csr_chunks"] == cr.size
+    assert np.array_equal(h.export("csr_chunk_row"), cr)
+    assert np.array_equal(h.export("csr_chunk_lo"), cl)
+    assert h.launches() == (1 + (2 if cr.size else 0) if A.n_rows else 0)
+    h.destroy()
+    x = matgen.vector(A.n_cols, 79, 1)
+    y0 = matgen.vector(A.n_rows, 79, 2)
+    for alpha, beta in ALPHA_BETA:
+        ref, bound = oracle.spmv_csr(A, x, alpha, beta, y0, with_bound=True)
+        h, out = run_format(sp, A, dA, "csr", torch.float64, alpha, beta, x, y0, csr_chunk=chunk)
+        ok, ratio, nbad = oracle.check_tolerance(out, ref, bound, TOL[torch.float64])
+        assert ok, f"{name} chunk={chunk} a={alpha} b={beta}: {nbad} bad rows, max ratio {ratio}"
+        h.destroy()
+    Ai = matgen.set_values(A, 991, "int")
+    dAi = to_dev(sp, Ai, torch.float32)
+    xi = matgen.vector(A.n_cols, 5, 1, "int")
+    yi = np.round(matgen.vector(A.n_rows, 5, 2, "f64") * 8)
+    ref = oracle.spmv_csr(Ai, xi, 2.0, -1.0, yi)
+    h, out = run_format(sp, Ai, dAi, "csr", torch.float32, 2.0, -1.0, xi, yi, csr_chunk=chunk)
+    assert np.array_equal(out, ref)
+    h.destroy()
+
+
+def test_csr_chunks_disabled_and_default(sp):
+    A = case("dense_row_1x5000", "f64")
+    dA = to_dev(sp, A, torch.float64)
+    assert sp.convert(dA, "csr", csr_chunk=-1).info()["csr_chunks"] == 0
+    assert sp.convert(dA, "csr").info()["csr_chunks"] == oracle.csr_chunks(A, 512)[0].size == 10   # default C = 512
+    assert sp.convert(dA, "csr_scalar", csr_chunk=7).info()["csr_chunks"] == 0

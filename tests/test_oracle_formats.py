@@ -414,3 +414,35 @@ def test_own_foreign_split_reassembles(P, compress):
         part = oracle.spmv_csr(foreign, xg, 1.5, 1.0, part)
         ok, ratio, _ = oracle.check_tolerance(part, ref[r0:r1], bound[r0:r1], 1e-13)
         assert ok, ratio
+
+
+# ------------------------------------------------------------------ CSR long-row chunks (A25)
+
+def test_csr_chunks_hand_example():
+    # row lengths 0, 5, 10, 3 with C = 2: rows longer than 4 are split into 2-nonzero chunks
+    A = matgen.from_lengths(np.array([0, 5, 10, 3]), 20, seed=3)
+    cr, cl = oracle.csr_chunks(A, 2)
+    assert cr.tolist() == [1, 1, 1, 2, 2, 2, 2, 2]
+    assert cl.tolist() == [0, 2, 4, 5, 7, 9, 11, 13]
+
+
+@pytest.mark.parametrize("C", [1, 2, 7, 64, 5000])
+def test_csr_chunks_tile_long_rows(C):
+    """Each long row's chunks tile [row_ptr[r], row_ptr[r+1]) in steps of C (last one
+    shorter), short rows have none, and summing the chunk partials reproduces the row."""
+    rng = np.random.default_rng(C)
+    for A in structured_cases():
+        cr, cl = oracle.csr_chunks(A, C)
+        lens = np.diff(A.row_ptr)
+        long_rows = np.nonzero(lens > 2 * C)[0]
+        assert cr.size == int(sum(-(-int(lens[r]) // C) for r in long_rows))
+        assert np.all(np.diff(cr) >= 0)
+        assert set(cr.tolist()) == set(long_rows.tolist())
+        x = rng.standard_normal(A.n_cols)
+        for r in long_rows:
+            sel = cr == r
+            lo = cl[sel]
+            a, b = int(A.row_ptr[r]), int(A.row_ptr[r + 1])
+            assert lo.tolist() == list(range(a, b, C))
+            parts = [np.sum(A.val[k:min(k + C, b)] * x[A.col[k:min(k + C, b)]]) for k in lo]
+            assert abs(sum(parts) - np.sum(A.val[a:b] * x[A.col[a:b]])) <= 1e-12 * np.sum(np.abs(A.val[a:b] * x[A.col[a:b]])) + 1e-300
