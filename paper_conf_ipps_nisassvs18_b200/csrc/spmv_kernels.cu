@@ -88,18 +88,28 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
             nlo = __ldg(rp + (nb + lane < n ? nb + lane : n));
             nhi = __ldg(rp + (nb + R < n ? nb + R : n));
         }
+        // group g owns the U consecutive rows g*U + u of the batch, so b[u] = a[u+1]:
+        // U + 1 shuffles of the batch's row pointers (a row per group slot u*G + g took 2U)
+        auto row_of = [&](int gg, int u) -> int { return gg * U + u; };
         IT a[U], b[U];
+        {
+            IT e[U + 1];
+#pragma unroll
+            for (int u = 0; u <= U; ++u) {
+                const int i = g * U + u;
+                const IT t = __shfl_sync(0xffffffffu, rp_lo, i & 31);
+                e[u] = i < R ? t : rp_hi;
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) { a[u] = e[u]; b[u] = e[u + 1]; }
+        }
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-            const int i = u * G + g;                         // row index within the batch
-            a[u] = __shfl_sync(0xffffffffu, rp_lo, i);
-            const IT nx = __shfl_sync(0xffffffffu, rp_lo, (i + 1) & 31);
-            b[u] = i + 1 < R ? nx : rp_hi;
-            if (base + i >= n) { a[u] = 0; b[u] = 0; }
+            if (base + row_of(g, u) >= n) { a[u] = 0; b[u] = 0; }
             if (CHUNKED && (int64_t)b[u] - (int64_t)a[u] > long_len) b[u] = a[u];   // chunked long row (A25): beta*y here
         }
-        // the y value this lane will write (writer lane sub == u of group g: row u*G + g)
-        const int64_t my_row = base + (int64_t)sub * G + g;
+        // the y value this lane will write (writer lane sub == u of group g: row row_of(g, u))
+        const int64_t my_row = base + row_of(g, sub < U ? sub : 0);
         const double yv = (!B0 && sub < U && my_row < n) ? (double)y[my_row] : 0.0;
         // first W elements of every row, all loads issued together
         int c0[U];
@@ -173,7 +183,7 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
                 for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
                 double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
                 part = warp_sum(tot + part);
-                const int writer = (i % G) * W + i / G;    // lane holding row i's group sum
+                const int writer = (i / U) * W + i % U;   // lane holding row i's group sum
                 if (lane == writer) mine += part;
             }
         }
@@ -1020,7 +1030,7 @@ spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col
     // W <= 8: 4 CTAs/SM (64 registers; LAP4096 0.442 -> 0.384 ms); wider groups keep
     // 3 CTAs/SM (80 registers; R-MAT 24 at W = 16: 4 CTAs/SM 11 % slower)
 #define SPMV_VEC(WW)                                                                                           \
-    if (long_len == INT64_MAX)                                                                                 \
+    if (long_len == INT64_MAX)                                                                            \
         k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false><<<g, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len); \
     else                                                                                                       \
         k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true><<<g, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len)
