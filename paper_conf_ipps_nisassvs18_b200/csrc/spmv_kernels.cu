@@ -372,16 +372,16 @@ __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wai
 // Returns R[l+1] (0 for lane 31) in *Rnext and R[l].
 __device__ __forceinline__ double seg_suffix(double head, bool flagged, double *Rnext) {
     const int lane = threadIdx.x & 31;
+    // At the round with offset o a lane has stopped iff a flagged lane lies in
+    // [lane, lane + o) or lane + o > 32 (induction over the rounds), so the stop state
+    // comes from one ballot instead of a shuffle per round; the sums are unchanged.
+    const unsigned fb = __ballot_sync(0xffffffffu, flagged);
     double R = head;
-    int F = flagged;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
         const double Rn = __shfl_down_sync(0xffffffffu, R, o);
-        const int Fn = __shfl_down_sync(0xffffffffu, F, o);
-        if (!F) {
-            if (lane + o < 32) { R += Rn; F = Fn; }
-            else F = 1;
-        }
+        const bool F = lane + o > 32 || ((fb >> lane) & ((1u << o) - 1u)) != 0u;
+        if (!F && lane + o < 32) R += Rn;
     }
     const double rn = __shfl_down_sync(0xffffffffu, R, 1);
     *Rnext = lane == 31 ? 0.0 : rn;
@@ -919,19 +919,8 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
     }
     if (kseg == 0) head = acc;
     // R[l] = head[l] + (lane l has a flag ? 0 : R[l+1])  (flag-segmented suffix sum)
-    double R = head;
-    bool F = kseg > 0;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const double Rn = __shfl_down_sync(0xffffffffu, R, o);
-        const int Fn = __shfl_down_sync(0xffffffffu, (int)F, o);
-        if (!F) {
-            if (lane + o < 32) { R += Rn; F = Fn; }
-            else F = true;
-        }
-    }
-    double Rnext = __shfl_down_sync(0xffffffffu, R, 1);
-    if (lane == 31) Rnext = 0.0;
+    double Rnext;
+    const double R = seg_suffix(head, kseg > 0, &Rnext);
     if (kseg > 0) emit(y_off + kseg - 1, acc + Rnext);
     if (lane == 0) {
         const bool lead = !(flag & 1u);
