@@ -482,6 +482,24 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
     double p[8];
 #pragma unroll
     for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
+    // rows past the window (sparse stretches: R-MAT's empty rows): the warp first writes
+    // beta*y to all of them, 128 rows per step, coalesced; the tile's segments there then
+    // add alpha*s (one more rounding of beta*y than the window path, within the bound)
+    if (!ACCUM && L > kOutWin) {
+        for (int64_t g0 = Wlo + kOutWin; g0 < Whi; g0 += kOutWin) {
+            double t4[kOutQ];
+#pragma unroll
+            for (int q = 0; q < kOutQ; ++q) {
+                const int64_t g = g0 + lane + 32 * q;
+                t4[q] = (!B0 && g < Whi) ? (double)y[g] : 0.0;
+            }
+#pragma unroll
+            for (int q = 0; q < kOutQ; ++q) {
+                const int64_t g = g0 + lane + 32 * q;
+                if (g < Whi) y[g] = B0 ? (V)0 : (V)(beta * t4[q]);
+            }
+        }
+    }
     __syncwarp();
 
     auto emit = [&](int64_t rr, double sum) {
@@ -489,10 +507,8 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
         if (li >= 0 && li < kOutWin) {
             s_acc[li] = sum;
             if (ACCUM) atomicOr(&s_mark[li >> 5], 1u << (li & 31));
-        } else if (ACCUM) {
-            y[rr] = (V)((double)y[rr] + alpha * sum);
         } else {
-            y_write<V, B0>(y, rr, sum, alpha, beta);
+            y[rr] = (V)((double)y[rr] + alpha * sum);
         }
     };
     int prev = __shfl_up_sync(0xffffffffu, r[7], 1);
@@ -506,8 +522,6 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
             if (r[s] != pr) {                                   // a segment (row) starts here
                 if (kseg == 0) head = acc;
                 else emit(cur, acc);                            // closed inside the lane
-                if (!ACCUM && pr >= 0 && (int64_t)r[s] - pr > 1) // empty rows beyond the window
-                    for (int64_t g = max((int64_t)pr + 1, Wlo + kOutWin); g < r[s]; ++g) y_beta<V, B0>(y, g, beta);
                 ++kseg;
                 cur = r[s];
                 acc = 0.0;
@@ -523,11 +537,6 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
         carry_row[t] = cont ? rf : -1;
         carry_val[t] = cont ? R : 0.0;
     }
-    if (!ACCUM && lane == last_lane) {                         // empty rows up to the next tile, beyond the window
-        for (int64_t g = max((int64_t)rl + 1, Wlo + kOutWin); g < nr; ++g) y_beta<V, B0>(y, g, beta);
-    }
-    if (!ACCUM && t == 0)                                      // leading empty rows beyond the window
-        for (int64_t g = kOutWin + lane; g < rf; g += 32) y_beta<V, B0>(y, g, beta);
     __syncwarp();
 #pragma unroll
     for (int q = 0; q < kOutQ; ++q) {
@@ -887,21 +896,19 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
     // empty window rows keep s = 0: y = alpha*0 + beta*y, as the definition (c1) reads
 #pragma unroll
     for (int q = 0; q < kQ; ++q) s_acc[wid][lane + 32 * q] = 0.0;
+    const unsigned flag = d & 0xFFFFu;
+    const int y_off = (int)((d >> 16) & 0x1FFu);
     double p[SIGMA];
 #pragma unroll
     for (int s = 0; s < SIGMA; ++s) p[s] = (double)v[s] * (double)ld_x(x + c[s], px);
     __syncwarp();
 
-    const unsigned flag = d & 0xFFFFu;
-    const int y_off = (int)((d >> 16) & 0x1FFu);
-    auto seg_row = [&](int idx) -> int64_t { return moff >= 0 ? __ldg(seg_map + moff + idx) : lo + idx; };
     auto emit = [&](int idx, double sum) {
-        const int64_t r = seg_row(idx);
-        const int64_t li = r - lo;
+        const int64_t li = moff >= 0 ? __ldg(seg_map + moff + idx) - lo : idx;
         if (li < kCsr5Win) {
             s_acc[wid][li] = sum;
         } else {
-            y_write<V, B0>(y, r, sum, alpha, beta);
+            y_write<V, B0>(y, lo + li, sum, alpha, beta);
         }
     };
 
@@ -938,9 +945,23 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
             y[lo + i] = (V)o;
         }
     }
-    if (L > kCsr5Win && moff >= 0) {                       // empty rows beyond the window
-        for (int64_t r = lo + kCsr5Win + lane; r < hi; r += 32)
-            if (__ldg(rp + r + 1) == __ldg(rp + r)) y_beta<V, B0>(y, r, beta);
+    if (L > kCsr5Win && moff >= 0) {
+        // empty rows past the window (sparse stretches: R-MAT's empty rows) get beta*y,
+        // 128 rows per step: their row pointers, then y, all loads of a step in flight
+        for (int64_t g0 = lo + kCsr5Win; g0 < hi; g0 += kCsr5Win) {
+            bool e[kQ];
+            double t4[kQ];
+#pragma unroll
+            for (int q = 0; q < kQ; ++q) {
+                const int64_t g = g0 + lane + 32 * q;
+                e[q] = g < hi && __ldg(rp + g + 1) == __ldg(rp + g);
+            }
+#pragma unroll
+            for (int q = 0; q < kQ; ++q) t4[q] = (!B0 && e[q]) ? (double)y[g0 + lane + 32 * q] : 0.0;
+#pragma unroll
+            for (int q = 0; q < kQ; ++q)
+                if (e[q]) y[g0 + lane + 32 * q] = B0 ? (V)0 : (V)(beta * t4[q]);
+        }
     }
 }
 
@@ -958,6 +979,15 @@ __global__ void k_fixup(const int64_t *__restrict__ carry_row, const double *__r
 }
 
 // ------------------------------------------------------------------ launch helpers
+
+// L1 / shared-memory split: the x gathers live in L1, so the tile kernels' shared memory
+// costs x hits.  SPMV_CARVEOUT=<percent> sets the preferred shared-memory carveout of
+// the tile kernels (experiments); unset = the driver's choice.
+template <typename K>
+void carveout(K *kernel) {
+    static const int pct = [] { const char *e = getenv("SPMV_CARVEOUT"); return e ? atoi(e) : -1; }();
+    if (pct >= 0) cudaFuncSetAttribute((const void *)kernel, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+}
 
 int grid_stride_blocks(const spmv_ctx *ctx, int64_t threads_needed, int per_sm) {
     int64_t g = ceil_div<int64_t>(threads_needed, kT);
@@ -1078,6 +1108,7 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
     }
     case SPMV_COO:
         if (h->nnz == 0) return launch_scale<V, B0>(h, y, beta, s);
+        carveout(k_coo<V, false, B0>);
         k_coo<V, false, B0><<<(unsigned)ceil_div<int64_t>(h->n_carry, kT / 32), kT, 0, s>>>(
             (const int *)h->arr[SPMV_ARR_COO_ROW].p, col, val, h->nnz, h->n_carry, x, y, n, alpha, beta, crow, cval);
         SPMV_LAUNCH_CHECK();
@@ -1095,6 +1126,7 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
             k_merge<V, IT, B0, 4, 6><<<g, kT, 0, s>>>(rp, col, val, cr, h->merge_tiles, dmax, x, y, alpha, beta, crow, cval);
         } else {
             const unsigned gp = (unsigned)std::min<int64_t>(g, (int64_t)h->ctx->sm_count * 3);
+            carveout(k_merge_persist<V, IT, B0, 8, 3>);
             k_merge_persist<V, IT, B0, 8, 3><<<gp, kT, 0, s>>>(rp, col, val, cr, h->merge_tiles, dmax, x, y, alpha, beta, crow, cval);
         }
     }
@@ -1104,6 +1136,7 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
         const int64_t warps = h->n_tiles + 1;
         const unsigned g = (unsigned)ceil_div<int64_t>(warps * 32, kT);
 #define SPMV_CSR5_LAUNCH(SG)                                                                                  \
+    carveout(k_csr5<SG, V, IT, B0>);                                                                          \
     k_csr5<SG, V, IT, B0><<<g, kT, 0, s>>>(rp, col, val, (const int64_t *)h->arr[SPMV_ARR_CSR5_TILE_PTR].p,   \
                                            (const int64_t *)h->arr[SPMV_ARR_CSR5_ROW_LO].p,                    \
                                            (const unsigned *)h->arr[SPMV_ARR_CSR5_TILE_DESC].p,                \

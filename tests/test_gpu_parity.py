@@ -61,6 +61,15 @@ def edge_cases(kind="f64"):
     cases["banded"] = matgen.window(3000, 3000, 9, 0.6, seed=9, mode=0, kind=kind)
     cases["blockdiag"] = matgen.window(2500, 4000, 64, 0.8, seed=10, mode=1, kind=kind)
     cases["poisson_rect"] = _lens_matrix(rng.poisson(20, 4000), 1500, 11, kind)
+    # mostly empty rows: COO / CSR5 / merge tiles spanning thousands of rows, with rows
+    # that have nonzeros past the tiles' 128-row output windows
+    lens = np.where(rng.random(60000) < 0.01, rng.integers(1, 9, 60000), 0)
+    cases["sparse_rows"] = _lens_matrix(lens, 60000, 13, kind)
+    # the same stretches between dense blocks (mean ~15: CSR5 sigma = 16, CSR W = 16)
+    lens = np.where(rng.random(60000) < 0.01, rng.integers(1, 9, 60000), 0)
+    lens[:20000] = 30
+    lens[40000:50000] = 30
+    cases["mixed_sparse"] = _lens_matrix(lens, 60000, 14, kind)
     zero = _lens_matrix(rng.integers(0, 9, 700), 700, 12, kind)
     cases["all_zero_vals"] = matgen.HostCSR(zero.row_ptr, zero.col, np.zeros(zero.nnz), zero.n_rows, zero.n_cols)
     return cases
@@ -77,7 +86,7 @@ def case(name, kind):
 
 CASE_NAMES = ["empty0x0", "1x1", "dense_row_1x5000", "col_n_x_1", "rect_3x7", "rect_7x3", "nnz0_rows5",
               "empty_runs", "long_row", "tile_bounds", "u2048", "lap37", "lap64", "rmat12", "rmat15",
-              "banded", "blockdiag", "poisson_rect", "all_zero_vals"]
+              "banded", "blockdiag", "poisson_rect", "all_zero_vals", "sparse_rows", "mixed_sparse"]
 
 
 def _guard(A, V):
@@ -142,7 +151,8 @@ def test_spmv_parity(sp, name, fmt, dtype):
         h.destroy()
 
 
-INT_CASES = ["rmat15", "lap64", "long_row", "tile_bounds", "empty_runs", "u2048", "poisson_rect", "dense_row_1x5000"]
+INT_CASES = ["rmat15", "lap64", "long_row", "tile_bounds", "empty_runs", "u2048", "poisson_rect", "dense_row_1x5000",
+             "sparse_rows", "mixed_sparse"]
 
 
 @pytest.mark.parametrize("dtype", [torch.float64, torch.float32], ids=["f64", "f32"])

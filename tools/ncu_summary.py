@@ -134,10 +134,12 @@ def full(rep, out, traffic=None, formats=("coo", "ell", "csr", "hyb", "merge", "
             fmt = "ell" if ("ell" in formats and seen[base] == 1) else "hyb"
         elif base == "k_csr_vector" and seen[base] == 1 and "csr" in formats:
             fmt = "csr"
+        elif base == "k_csr_chunks" and "csr" in formats:
+            fmt = "csr"
         if fmt:
             rd = to_bytes(d["dram__bytes_read.sum"], units[hdr.index("dram__bytes_read.sum")])
             wr = to_bytes(d["dram__bytes_write.sum"], units[hdr.index("dram__bytes_write.sum")])
-            if fmt == "hyb" or fmt not in trafficmap:
+            if fmt == "hyb" or fmt not in trafficmap or base == "k_csr_chunks":
                 trafficmap[fmt] = trafficmap.get(fmt, 0) + rd + wr
     with open(out, "w") as f:
         f.write("\n".join(lines) + "\n")
