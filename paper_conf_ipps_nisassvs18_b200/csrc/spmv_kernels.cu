@@ -641,15 +641,24 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
         const int i = lane + 32 * q;
         yv[q] = (!B0 && i < nrows) ? (double)y[r0 + i] : 0.0;
     }
-    for (int i = lane; i < nrows; i += 32) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
-    const bool r0_inside = (int64_t)__ldg(rp + r0) == k0;   // A7: rp[r0] <= k0 always
+    // the tile's row ends (first 64 in registers) are issued with the chunk loads and
+    // stored to shared memory only after the x gathers are in flight
+    const IT re0 = lane < nrows ? __ldg(rp + r0 + 1 + lane) : (IT)0;
+    const IT re1 = lane + 32 < nrows ? __ldg(rp + r0 + 33 + lane) : (IT)0;
+    const IT rp0 = __ldg(rp + r0);
     // segment-start flags, one byte per chunk position (plain stores, no atomics)
     unsigned char *s_fb = reinterpret_cast<unsigned char *>(s_flag);
     for (int i = lane; i < TI / 8 + 1; i += 32) s_flag[i] = make_uint2(0u, 0u);
+    double xg[LI];
+#pragma unroll
+    for (int e = 0; e < LI; ++e) xg[e] = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)ld_x(x + c[e], px) : 0.0;
+    if (lane < nrows) s_end[lane] = (int)((int64_t)re0 - k0);
+    if (lane + 32 < nrows) s_end[lane + 32] = (int)((int64_t)re1 - k0);
+    for (int i = lane + 64; i < nrows; i += 32) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
+    const bool r0_inside = (int64_t)rp0 == k0;               // A7: rp[r0] <= k0 always
     double p[LI];
 #pragma unroll
-    for (int e = 0; e < LI; ++e)
-        p[e] = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)v[e] * (double)ld_x(x + c[e], px) : 0.0;
+    for (int e = 0; e < LI; ++e) p[e] = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)v[e] * xg[e] : 0.0;
     __syncwarp();
     // segment starts: local row i (1 <= i <= nrows) starts at s_end[i-1]; row 0 at 0 if
     // r0_inside.  The bitmap is indexed by chunk position (tile position + off).
@@ -966,15 +975,50 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
 }
 
 // ------------------------------------------------------------------ fix-up (G13)
+// Carries are stored in tile order, so a row's carries are one contiguous run (a row
+// spanning many tiles -- an R-MAT hub row -- gives a run of hundreds).  One warp per 32
+// consecutive carries: a flag-segmented suffix sum gives each run's sum inside the
+// chunk; the run's head lane adds alpha * sum to y.  A run that starts in the chunk and
+// reaches its end is continued by the whole warp, 32 carries per step (coalesced loads,
+// warp sums, added in chunk order), so no thread walks a long run serially.  Runs that
+// began in an earlier chunk are left to the warp holding their head.
 template <typename V>
 __global__ void k_fixup(const int64_t *__restrict__ carry_row, const double *__restrict__ carry_val, int64_t n,
                         V *__restrict__ y, double alpha) {
-    for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t r = carry_row[c];
-        if (r < 0 || (c > 0 && carry_row[c - 1] == r)) continue;
-        double s = 0.0;
-        for (int64_t q = c; q < n && carry_row[q] == r; ++q) s += carry_val[q];
-        y[r] = (V)((double)y[r] + alpha * s);
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * 32 < n; w += nw) {
+        const int64_t c = w * 32 + lane;
+        const int64_t key = c < n ? carry_row[c] : -1;
+        const double val = c < n ? carry_val[c] : 0.0;
+        const int64_t prev = w > 0 ? carry_row[w * 32 - 1] : -1;
+        const int64_t kup = __shfl_up_sync(0xffffffffu, key, 1);
+        const int64_t kdn = __shfl_down_sync(0xffffffffu, key, 1);
+        const bool head = lane == 0 ? key != prev : key != kup;
+        const bool last = lane == 31 || key != kdn;            // run ends at this lane (inside the chunk)
+        double Rnext;
+        const double R = seg_suffix(val, last, &Rnext);        // R[l] = val[l] + (last[l] ? 0 : R[l+1])
+        // the chunk's final run may continue into the next chunks
+        const int64_t k31 = __shfl_sync(0xffffffffu, key, 31);
+        const bool open = k31 >= 0 && (w + 1) * 32 < n && carry_row[(w + 1) * 32] == k31;
+        const unsigned hb = __ballot_sync(0xffffffffu, head && key == k31);
+        const int h31 = 31 - __clz(hb);                        // head lane of the final run
+        const bool own_final = open && hb != 0u && !(h31 == 0 && k31 == prev);
+        double tail = 0.0;
+        if (own_final) {                                        // warp-uniform
+            for (int64_t q = (w + 1) * 32; q < n; q += 32) {
+                const int64_t kq = q + lane < n ? carry_row[q + lane] : -1;
+                const double vq = q + lane < n ? carry_val[q + lane] : 0.0;
+                const unsigned m = __ballot_sync(0xffffffffu, kq == k31);
+                const unsigned pre = ~m ? ((1u << __ffs(~m) - 1) - 1u) : 0xffffffffu;   // leading run of equal keys
+                tail += warp_sum((pre >> lane) & 1u ? vq : 0.0);
+                if (pre != 0xffffffffu) break;
+            }
+        }
+        if (head && key >= 0 && !(lane == 0 && key == prev)) {
+            const double sum = (lane == h31 && own_final) ? R + tail : R;
+            y[key] = (V)((double)y[key] + alpha * sum);
+        }
     }
 }
 
@@ -1006,7 +1050,7 @@ spmv_status launch_scale(spmv_handle *h, V *y, double beta, cudaStream_t s) {
 template <typename V>
 spmv_status launch_fixup(spmv_handle *h, V *y, double alpha, cudaStream_t s) {
     if (h->n_carry == 0) return SPMV_OK;
-    k_fixup<V><<<grid_stride_blocks(h->ctx, h->n_carry, 16), kT, 0, s>>>(
+    k_fixup<V><<<grid_stride_blocks(h->ctx, ceil_div<int64_t>(h->n_carry, 32) * 32, 16), kT, 0, s>>>(
         (const int64_t *)h->carry_row.p, (const double *)h->carry_val.p, h->n_carry, y, alpha);
     SPMV_LAUNCH_CHECK();
     return SPMV_OK;

@@ -101,10 +101,11 @@ def lib():
     """Load libspmv.so; fails loudly if it was not built (no fallback)."""
     global _lib
     if _lib is None:
-        if not os.path.exists(LIB_PATH):
-            raise RuntimeError(f"{LIB_PATH} is missing: build it with __graft_entry__.build() "
+        path = os.environ.get("SPMV_LIB_PATH", LIB_PATH)   # A/B experiments (tools/): another build
+        if not os.path.exists(path):
+            raise RuntimeError(f"{path} is missing: build it with __graft_entry__.build() "
                                "(there is no CPU fallback)")
-        L = C.CDLL(LIB_PATH)
+        L = C.CDLL(path)
         sig = {
             "spmv_abi_version": (C.c_int, []),
             "spmv_init": (C.c_int, [C.c_int, C.POINTER(spmv_allocator), C.POINTER(_P)]),
