@@ -522,3 +522,46 @@ def test_csr_chunks_disabled_and_default(sp):
     assert sp.convert(dA, "csr", csr_chunk=-1).info()["csr_chunks"] == 0
     assert sp.convert(dA, "csr").info()["csr_chunks"] == oracle.csr_chunks(A, 512)[0].size == 10   # default C = 512
     assert sp.convert(dA, "csr_scalar", csr_chunk=7).info()["csr_chunks"] == 0
+
+
+# ------------------------------------------------------------------ configs[2] at full size
+
+def _rmat24():
+    if "rmat" not in _BIG:
+        _BIG["rmat"] = matgen.rmat(24)
+    return _BIG["rmat"]
+
+
+RMAT_FORMATS = ("coo", "csr", "hyb", "merge", "csr5")   # ELL is infeasible (A4)
+
+
+def test_full_size_rmat24(sp):
+    """BASELINE configs[2] (R-MAT scale 24, 2.6e8 nonzeros, 56% empty rows, a 190K-nonzero
+    hub row) at full size in bench.py's launch configuration: features bit-exact; fp64
+    alpha = beta = 1 within the A16 bound on every row; the integer regime (fp32 storage,
+    alpha = 2, beta = -1) bit-exact on every row, for every feasible format."""
+    A = _rmat24()
+    dA = sp.CSR.from_host(A, dtype=torch.float64)
+    f, fo = sp.features(dA), oracle.features(A)
+    assert all(f[k] == fo[k] for k in sp.PAPER_FEATURES)
+    with pytest.raises(sp.SpmvError) as e:
+        sp.convert(dA, "ell")
+    assert e.value.status == 3
+    x = matgen.vector(A.n_cols, matgen.SEEDS["rmat24"], 1)
+    y0 = matgen.vector(A.n_rows, matgen.SEEDS["rmat24"], 2)
+    ref, bound = oracle.spmv_csr(A, x, 1.0, 1.0, y0, with_bound=True)
+    for fmt in RMAT_FORMATS:
+        h, out = run_format(sp, A, dA, fmt, torch.float64, 1.0, 1.0, x, y0)
+        ok, ratio, nbad = oracle.check_tolerance(out, ref, bound, 1e-12)
+        h.destroy()
+        assert ok, (fmt, nbad, ratio)
+    del dA, ref, bound
+    Ai = matgen.set_values(A, 991, "int")
+    dAi = sp.CSR.from_host(Ai, dtype=torch.float32)
+    xi = matgen.vector(A.n_cols, 5, 1, "int")
+    yi = np.round(matgen.vector(A.n_rows, 5, 2, "f64") * 8)
+    refi = oracle.spmv_csr(Ai, xi, 2.0, -1.0, yi)
+    for fmt in RMAT_FORMATS:
+        h, out = run_format(sp, Ai, dAi, fmt, torch.float32, 2.0, -1.0, xi, yi)
+        h.destroy()
+        assert np.array_equal(out, refi), fmt
