@@ -641,24 +641,15 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
         const int i = lane + 32 * q;
         yv[q] = (!B0 && i < nrows) ? (double)y[r0 + i] : 0.0;
     }
-    // the tile's row ends (first 64 in registers) are issued with the chunk loads and
-    // stored to shared memory only after the x gathers are in flight
-    const IT re0 = lane < nrows ? __ldg(rp + r0 + 1 + lane) : (IT)0;
-    const IT re1 = lane + 32 < nrows ? __ldg(rp + r0 + 33 + lane) : (IT)0;
-    const IT rp0 = __ldg(rp + r0);
+    for (int i = lane; i < nrows; i += 32) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
+    const bool r0_inside = (int64_t)__ldg(rp + r0) == k0;   // A7: rp[r0] <= k0 always
     // segment-start flags, one byte per chunk position (plain stores, no atomics)
     unsigned char *s_fb = reinterpret_cast<unsigned char *>(s_flag);
     for (int i = lane; i < TI / 8 + 1; i += 32) s_flag[i] = make_uint2(0u, 0u);
-    double xg[LI];
-#pragma unroll
-    for (int e = 0; e < LI; ++e) xg[e] = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)ld_x(x + c[e], px) : 0.0;
-    if (lane < nrows) s_end[lane] = (int)((int64_t)re0 - k0);
-    if (lane + 32 < nrows) s_end[lane + 32] = (int)((int64_t)re1 - k0);
-    for (int i = lane + 64; i < nrows; i += 32) s_end[i] = (int)((int64_t)__ldg(rp + r0 + 1 + i) - k0);
-    const bool r0_inside = (int64_t)rp0 == k0;               // A7: rp[r0] <= k0 always
     double p[LI];
 #pragma unroll
-    for (int e = 0; e < LI; ++e) p[e] = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)v[e] * xg[e] : 0.0;
+    for (int e = 0; e < LI; ++e)
+        p[e] = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)v[e] * (double)ld_x(x + c[e], px) : 0.0;
     __syncwarp();
     // segment starts: local row i (1 <= i <= nrows) starts at s_end[i-1]; row 0 at 0 if
     // r0_inside.  The bitmap is indexed by chunk position (tile position + off).

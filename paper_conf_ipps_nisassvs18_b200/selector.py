@@ -165,6 +165,7 @@ def evaluate(X: np.ndarray, y: np.ndarray, T: np.ndarray, model: str, seed: int 
     return {"model": model, "n": int(len(y)), "params": params,
             "cv_acc_mean": float(cv_acc.mean()), "cv_acc_std": float(cv_acc.std()),
             "test_acc": float(np.mean(pred == y[te])), "test_n": int(len(te)),
+            "test_acc_within_2pct": float(np.mean(sd <= 1.02)), "test_acc_within_5pct": float(np.mean(sd <= 1.05)),
             "slowdown_hist": slowdown_histogram(sd),
             "mean_slowdown_mispredicted": float(np.mean(wrong)) if len(wrong) else 1.0,
             "geo_mean_slowdown_all": float(np.exp(np.mean(np.log(np.minimum(sd, 1e6)))))}
@@ -268,7 +269,8 @@ def _main():
         with open(a.out, "w") as fh:
             fh.write(txt + "\n")
     for k, v in res["classification"].items():
-        print(f"{k:28s} cv {v['cv_acc_mean']:.3f}  test {v['test_acc']:.3f}  slowdown {v['slowdown_hist']}")
+        print(f"{k:28s} cv {v['cv_acc_mean']:.3f}  test {v['test_acc']:.3f}  (<=2%: {v['test_acc_within_2pct']:.3f})  "
+              f"slowdown {v['slowdown_hist']}")
     for f, v in res["regression"]["formats"].items():
         print(f"RME {f:6s} mlp {v['rme_mlp']:.3f}  ensemble {v['rme_mlp_ensemble']:.3f}")
     print("indirect", res["regression"]["indirect_mlp_ensemble"])
