@@ -22,9 +22,11 @@ def main():
     src = hdr.index("Source")
     recs = []
     tot = 0
+    seen = set()
     for r in rows[hi + 1:]:
-        if len(r) <= si:
+        if len(r) <= si or r[0] in seen:      # one launch: each address once
             continue
+        seen.add(r[0])
         try:
             v = float(r[si])
         except ValueError:
