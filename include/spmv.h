@@ -214,7 +214,12 @@ typedef enum {
     SPMV_ARR_CSR5_MAP_OFF = 13,     /* int64 [tiles] (-1 = no empty row in range) */
     SPMV_ARR_CSR5_SEG_MAP = 14,     /* int64 [map_len] */
     SPMV_ARR_CSR_CHUNK_ROW = 15,    /* CSR: int64 [chunks], row of each long-row chunk (A25) */
-    SPMV_ARR_CSR_CHUNK_LO = 16      /* CSR: int64 [chunks], first nonzero of each chunk      */
+    SPMV_ARR_CSR_CHUNK_LO = 16,     /* CSR: int64 [chunks], first nonzero of each chunk      */
+    SPMV_ARR_MERGE_TILE_CLASS = 17, /* MERGE: uint8 [tiles], 1 = row-sum tile (A28): fewer than
+                                       64 row ends in the tile and every row's part inside the
+                                       tile (the open row included) <= 32 nonzeros; else 0     */
+    SPMV_ARR_MERGE_TILE_ORDER = 18  /* MERGE: int32 [tiles], the tile ids stably partitioned by
+                                       class: class-1 tiles first (ascending), then class 0    */
 } spmv_array_id;
 
 /* Copy array `id` of the handle to host memory (blocking on `stream`).

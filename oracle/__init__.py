@@ -79,6 +79,7 @@ def lib():
             "ora_merge_ntiles": (_i64, [_i64, _i64, _i64]),
             "ora_csr_chunks": (_i64, [_i64, _p, _i64, _p, _p]),
             "ora_merge_coords": (C.c_int, [_i64, _p, _i64, _p, _p]),
+            "ora_merge_class": (C.c_int, [_i64, _p, _i64, _i64, _i64, _p]),
             "ora_csr5_sigma": (_i64, [_i64, _i64]),
             "ora_csr5_map_len": (_i64, [_i64, _p, _i64]),
             "ora_csr5_encode": (C.c_int, [_i64, _p, _p, _p, _i64, C.c_int,
@@ -222,6 +223,16 @@ def merge_coords(A, T):
     rc = lib().ora_merge_coords(A.n_rows, _ptr(A.row_ptr), int(T), _ptr(cr), _ptr(cn))
     assert rc == 0
     return cr, cn
+
+
+def merge_class(A, T, max_rows=64, max_len=32):
+    """Merge tile class (A28): uint8 per tile, 1 = row-sum tile."""
+    A = CSR.of(A)
+    nt = int(lib().ora_merge_ntiles(A.n_rows, A.nnz, int(T)))
+    cls = _buf(nt, np.uint8)
+    rc = lib().ora_merge_class(A.n_rows, _ptr(A.row_ptr), int(T), int(max_rows), int(max_len), _ptr(cls))
+    assert rc == 0
+    return cls
 
 
 def csr_chunks(A, C):

@@ -243,6 +243,30 @@ int ora_merge_coords(int64_t n_rows, const int64_t *row_ptr, int64_t T,
     return t == n_tiles + 1 ? 0 : -2;
 }
 
+/* A28: class of merge tile t = 1 iff the tile consumes fewer than
+ * max_rows row ends and no row receives more than max_len of the tile's nonzeros
+ * (the row still open at the tile's end included).  Walks the merge path item by
+ * item, counting the nonzeros the current row takes inside the current tile. */
+int ora_merge_class(int64_t n_rows, const int64_t *row_ptr, int64_t T,
+                    int64_t max_rows, int64_t max_len, uint8_t *cls)
+{
+    int64_t nnz = row_ptr[n_rows];
+    int64_t total = n_rows + nnz;
+    int64_t n_tiles = ora_merge_ntiles(n_rows, nnz, T);
+    if (n_tiles < 0) return -1;
+    int64_t i = 0, j = 0;
+    for (int64_t t = 0; t < n_tiles; ++t) {
+        int64_t d_end = (t + 1) * T < total ? (t + 1) * T : total;
+        int64_t ends = 0, run = 0, run_max = 0;
+        for (int64_t d = t * T; d < d_end; ++d) {
+            if (i < n_rows && row_ptr[i + 1] <= j) { ++i; ++ends; run = 0; }
+            else { ++j; ++run; if (run > run_max) run_max = run; }
+        }
+        cls[t] = (ends < max_rows && run_max <= max_len) ? 1 : 0;
+    }
+    return 0;
+}
+
 /* ------------------------------------------------------------------ CSR5 */
 
 #define ORA_OMEGA 32

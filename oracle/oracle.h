@@ -75,6 +75,10 @@ int ora_csr2hyb(int64_t n_rows, const int64_t *row_ptr, const int32_t *col,
 int64_t ora_merge_ntiles(int64_t n_rows, int64_t nnz, int64_t T);
 int ora_merge_coords(int64_t n_rows, const int64_t *row_ptr, int64_t T,
                      int64_t *coord_row, int64_t *coord_nz);
+/* Merge tile class (A28): cls[t] = 1 iff tile t consumes fewer than max_rows row
+ * ends and no row takes more than max_len of its nonzeros (walk, as above). */
+int ora_merge_class(int64_t n_rows, const int64_t *row_ptr, int64_t T,
+                    int64_t max_rows, int64_t max_len, uint8_t *cls);
 
 /* CSR long-row chunks (A25): a row with len > 2*C is reduced as
  * ceil(len/C) chunks of C nonzeros (the last one shorter), chunk j of row r starting at

@@ -255,8 +255,9 @@ spmv_status spmv_info(const spmv_handle *h, spmv_handle_info *o) {
     size_t dev = 0, fmt_bytes = 0;
     for (int i = 0; i < kMaxArrays; ++i) {
         if (h->arr[i].owned) dev += h->arr[i].bytes;
-        // the merge kernel derives the nonzero coordinate as d - row (A7): kept for export, not read
-        if (i != SPMV_ARR_MERGE_COORD_NZ) fmt_bytes += h->arr[i].bytes;
+        // the merge kernels derive the nonzero coordinate as d - row (A7) and take the tile
+        // class from the tile order: both kept for export, not read by a run
+        if (i != SPMV_ARR_MERGE_COORD_NZ && i != SPMV_ARR_MERGE_TILE_CLASS) fmt_bytes += h->arr[i].bytes;
     }
     dev += h->carry_row.bytes + h->carry_val.bytes;
     o->device_bytes = dev;
@@ -285,7 +286,8 @@ spmv_status spmv_export(const spmv_handle *h, spmv_array_id id, void *dst, size_
         case SPMV_HYB: present = id == SPMV_ARR_ELL_COL || id == SPMV_ARR_ELL_VAL || id == SPMV_ARR_COO_ROW ||
                                  id == SPMV_ARR_HYB_COO_COL || id == SPMV_ARR_HYB_COO_VAL; break;
         case SPMV_MERGE: present = id <= SPMV_ARR_VAL || id == SPMV_ARR_MERGE_COORD_ROW ||
-                                   id == SPMV_ARR_MERGE_COORD_NZ; break;
+                                   id == SPMV_ARR_MERGE_COORD_NZ || id == SPMV_ARR_MERGE_TILE_CLASS ||
+                                   id == SPMV_ARR_MERGE_TILE_ORDER; break;
         case SPMV_CSR5: present = id <= SPMV_ARR_VAL || (id >= SPMV_ARR_CSR5_TILE_PTR && id <= SPMV_ARR_CSR5_SEG_MAP); break;
         }
         if (!present) { set_error("handle has no such array"); return SPMV_ERR_INVALID_ARG; }

@@ -119,6 +119,36 @@ __global__ void k_merge_coords(const IT *rp, int64_t n, int64_t nnz, int64_t T, 
     }
 }
 
+// merge tile class (A28): 1 = row-sum tile -- fewer than kMergeLeanRows row ends and
+// every in-tile row part (row r1's included) <= kMergeLeanLen nonzeros.  Row i's part
+// is clip(rp[i+1]) - clip(rp[i]), clip to the tile's nonzero range [k0, k1].
+template <typename IT>
+__global__ void k_merge_class(const IT *rp, int64_t n, const int64_t *crow, const int64_t *cnz, int64_t tiles,
+                              unsigned char *cls) {
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < tiles; t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r0 = crow[t], r1 = crow[t + 1], k0 = cnz[t], k1 = cnz[t + 1];
+        bool ok = r1 - r0 < kMergeLeanRows;
+        int64_t lo = k0;                                  // clip(rp[r0]) = k0 (A7: rp[r0] <= k0)
+        for (int64_t i = r0; ok && i <= r1; ++i) {
+            int64_t hi = i < n ? (int64_t)rp[i + 1] : k1;
+            hi = hi < k0 ? k0 : hi > k1 ? k1 : hi;
+            ok = hi - lo <= kMergeLeanLen;
+            lo = hi;
+        }
+        cls[t] = ok ? 1 : 0;
+    }
+}
+__global__ void k_u8_to_i64(const unsigned char *a, int64_t n, int64_t *b) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        b[i] = a[i] != 0;
+}
+// stable partition of the tile ids by class (class 1 first); pre = exclusive prefix
+// count of class-1 tiles, nl = their total
+__global__ void k_merge_order(const unsigned char *cls, const int64_t *pre, int64_t tiles, int64_t nl, int *order) {
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < tiles; t += (int64_t)gridDim.x * blockDim.x)
+        order[cls[t] ? pre[t] : nl + (t - pre[t])] = (int)t;
+}
+
 // ---- CSR5 (encoding A6) -----------------------------------
 
 template <typename IT>
@@ -418,6 +448,10 @@ spmv_status convert_t(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, const s
             return SPMV_ERR_UNSUPPORTED;
         }
         int64_t tiles = ceil_div<int64_t>(n + nnz, T);
+        if (tiles >= INT32_MAX) {   // the tile order is int32
+            set_error("too many merge tiles");
+            return SPMV_ERR_SIZE;
+        }
         h->merge_T = T;
         h->merge_tiles = tiles;
         SPMV_TRY(arr_alloc(h, SPMV_ARR_MERGE_COORD_ROW, (tiles + 1) * 8, s));
@@ -426,6 +460,31 @@ spmv_status convert_t(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, const s
             rp, n, nnz, T, tiles, (int64_t *)h->arr[SPMV_ARR_MERGE_COORD_ROW].p,
             (int64_t *)h->arr[SPMV_ARR_MERGE_COORD_NZ].p);
         SPMV_LAUNCH_CHECK();
+        SPMV_TRY(arr_alloc(h, SPMV_ARR_MERGE_TILE_CLASS, tiles, s));
+        h->merge_lean = 0;
+        if (tiles > 0) {
+            k_merge_class<IT><<<grid_cap(ctx, tiles), kT, 0, s>>>(
+                rp, n, (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_ROW].p,
+                (const int64_t *)h->arr[SPMV_ARR_MERGE_COORD_NZ].p, tiles,
+                (unsigned char *)h->arr[SPMV_ARR_MERGE_TILE_CLASS].p);
+            SPMV_LAUNCH_CHECK();
+            Scratch c64(ctx, s), pre(ctx, s);
+            SPMV_TRY(c64.alloc(tiles * 8));
+            SPMV_TRY(pre.alloc((tiles + 1) * 8));
+            k_u8_to_i64<<<grid_cap(ctx, tiles), kT, 0, s>>>((const unsigned char *)h->arr[SPMV_ARR_MERGE_TILE_CLASS].p,
+                                                            tiles, c64.as<int64_t>());
+            SPMV_LAUNCH_CHECK();
+            SPMV_TRY(exclusive_scan_i64(ctx, c64.as<int64_t>(), pre.as<int64_t>(), tiles, s));
+            int64_t nl = 0;
+            SPMV_CUDA_TRY(cudaMemcpyAsync(&nl, pre.as<int64_t>() + tiles, 8, cudaMemcpyDeviceToHost, s));
+            SPMV_CUDA_TRY(cudaStreamSynchronize(s));
+            SPMV_TRY(arr_alloc(h, SPMV_ARR_MERGE_TILE_ORDER, tiles * 4, s));
+            k_merge_order<<<grid_cap(ctx, tiles), kT, 0, s>>>((const unsigned char *)h->arr[SPMV_ARR_MERGE_TILE_CLASS].p,
+                                                              pre.as<int64_t>(), tiles, nl,
+                                                              (int *)h->arr[SPMV_ARR_MERGE_TILE_ORDER].p);
+            SPMV_LAUNCH_CHECK();
+            h->merge_lean = (int64_t)nl;
+        }
         h->n_carry = tiles;
         break;
     }

@@ -28,7 +28,8 @@ constexpr int kT = kRunThreads;
 constexpr int kIPT = kItemsPerThread;
 constexpr int kWIPT = kWarpItemsPerLane;
 constexpr int kMinBlocks = 4;   // 4 CTAs x 256 threads per SM: <= 64 registers
-constexpr int kFold = 256;   // sequential steps per accumulator before folding (A13)
+constexpr int kFold = 256;
+constexpr int kMergeRowsMB = 4;   // k_merge_rows CTAs per SM   // sequential steps per accumulator before folding (A13)
 
 // ------------------------------------------------------------------ helpers
 
@@ -772,36 +773,206 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
                               px);
 }
 
-// persistent: warp w takes tiles w, w + W, ...; the next tile's coordinates are loaded
-// while the current one is processed (hides the coordinate -> nonzero load dependency)
-template <typename V, typename IT, bool B0, int LI, int MB>
+// row-pointer entry through a volatile load, so that it is issued where it is written
+// (beside the tile's chunk loads) and not sunk behind the x gathers
+__device__ __forceinline__ int64_t ld_rp(const int *p) {
+    int v;
+    asm volatile("ld.global.nc.s32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ int64_t ld_rp(const int64_t *p) {
+    int64_t v;
+    asm volatile("ld.global.nc.s64 %0, [%1];" : "=l"(v) : "l"(p));
+    return v;
+}
+
+// Persistent warps over positions [i0, i1) of the tile order (A28): warp w takes
+// positions i0 + w, i0 + w + W, ...  Two-stage prefetch: while tile order[i] runs, the
+// coordinates of order[i + W] and the id order[i + 2W] are in flight.
+#define SPMV_MERGE_SCHEDULE(BODY)                                                                        \
+    const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;                                          \
+    int64_t i = i0 + ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);                         \
+    if (i >= i1) return;                                                                               \
+    int64_t t = __ldg(order + i);                                                                      \
+    int64_t r0 = ld_coord(crow + t, px), r1 = ld_coord(crow + t + 1, px);                              \
+    int64_t tb = i + W < i1 ? __ldg(order + i + W) : 0;                                                \
+    while (true) {                                                                                     \
+        int64_t q0 = 0, q1 = 0, tc = 0;                                                                \
+        if (i + W < i1) { q0 = ld_coord(crow + tb, px); q1 = ld_coord(crow + tb + 1, px); }            \
+        if (i + 2 * W < i1) tc = __ldg(order + i + 2 * W);                                             \
+        BODY;                                                                                          \
+        i += W;                                                                                        \
+        if (i >= i1) break;                                                                            \
+        t = tb; r0 = q0; r1 = q1; tb = tc;                                                             \
+        __syncwarp();                                                                                  \
+    }
+
+// Segmented-sum tiles (any class).  LIST = false: tiles i0 + w, i0 + w + W, ... (the
+// next tile's coordinates loaded while the current one runs); LIST = true: positions
+// [i0, i1) of the tile order.
+template <typename V, typename IT, bool B0, int LI, int MB, bool LIST>
 __global__ void __launch_bounds__(kT, MB)
 k_merge_persist(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
-                const int64_t *__restrict__ crow, int64_t n_tiles, int64_t dmax,
-                const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
+                const int64_t *__restrict__ crow, const int *__restrict__ order, int64_t i0, int64_t i1,
+                int64_t dmax, const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
                 int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
     constexpr int TI = 32 * LI;
     __shared__ double s_sum_all[kT / 32][TI];
     __shared__ int s_end_all[kT / 32][TI];
     __shared__ uint2 s_flag_all[kT / 32][TI / 8 + 1];
     const int wid = threadIdx.x >> 5;
-    const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    if (t >= n_tiles) return;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
-    int64_t r0 = ld_coord(crow + t, px), r1 = ld_coord(crow + t + 1, px);
-    while (true) {
-        const int64_t tn = t + W;
-        int64_t q0 = 0, q1 = 0;
-        if (tn < n_tiles) { q0 = ld_coord(crow + tn, px); q1 = ld_coord(crow + tn + 1, px); }
-        merge_tile<V, IT, B0, LI>(rp, col, val, t, r0, r1, merge_k(t, TI, r0, dmax), merge_k(t + 1, TI, r1, dmax), x,
-                                  y, alpha, beta, carry_row, carry_val, s_sum_all[wid], s_end_all[wid],
-                                  s_flag_all[wid], pa, px);
-        if (tn >= n_tiles) break;
-        t = tn; r0 = q0; r1 = q1;
-        __syncwarp();
+    auto body = [&](int64_t t, int64_t r0, int64_t r1) {
+        merge_tile<V, IT, B0, LI>(rp, col, val, t, r0, r1, merge_k(t, TI, r0, dmax), merge_k(t + 1, TI, r1, dmax), x, y,
+                                  alpha, beta, carry_row, carry_val, s_sum_all[wid], s_end_all[wid], s_flag_all[wid],
+                                  pa, px);
+    };
+    if constexpr (!LIST) {
+        const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+        int64_t t = i0 + ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+        if (t >= i1) return;
+        int64_t r0 = ld_coord(crow + t, px), r1 = ld_coord(crow + t + 1, px);
+        while (true) {
+            const int64_t tn = t + W;
+            int64_t q0 = 0, q1 = 0;
+            if (tn < i1) { q0 = ld_coord(crow + tn, px); q1 = ld_coord(crow + tn + 1, px); }
+            body(t, r0, r1);
+            if (tn >= i1) break;
+            t = tn; r0 = q0; r1 = q1;
+            __syncwarp();
+        }
+    } else {
+        SPMV_MERGE_SCHEDULE(body(t, r0, r1))
     }
 }
+
+// Class-1 (row-sum) tile, A28: fewer than 64 row ends and every in-tile row part <= 32
+// nonzeros.  Lane l holds its 32-byte aligned chunk of 8 nonzeros (as merge_tile; loaded
+// one tile ahead by the caller) and loads the ends of rows l and l + 32; the products go
+// to shared memory in chunk order and lane i sums rows i and i + 32 sequentially (two
+// accumulators) -- no segment flags, no cross-lane segmented scan.  Row i covers local
+// positions [end(i-1), end(i)) (row 0 from 0: the earlier parts of a row begun in an
+// earlier tile arrive as carries); row nrows is the open row r1, its part the tile carry.
+template <typename V>
+struct MergeChunk {
+    int c[8];
+    V v[8];
+};
+template <typename V>
+__device__ __forceinline__ void merge_chunk_load(const int *__restrict__ col, const V *__restrict__ val, int64_t k0,
+                                                 int64_t k1, MergeChunk<V> &ch, uint64_t pa) {
+    const int lane = threadIdx.x & 31;
+    const int off = (int)(k0 & 7);
+    if (lane * 8 - off < (int)(k1 - k0)) {
+        ld256(col + (k0 - off) + lane * 8, ch.c, pa);
+        VecLoad8<V>::load(val + (k0 - off) + lane * 8, ch.v, pa);
+    }
+}
+
+template <typename V, typename IT, bool B0>
+__device__ __forceinline__ void
+merge_rows_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val, int64_t t,
+                int64_t r0, int64_t r1, int64_t k0, int64_t k1, const MergeChunk<V> &ch, const V *__restrict__ x,
+                V *__restrict__ y, double alpha, double beta, int64_t *__restrict__ carry_row,
+                double *__restrict__ carry_val, double *s_p, uint64_t pa, uint64_t px) {
+    constexpr int LI = 8;
+    const int lane = threadIdx.x & 31;
+    const int nrows = (int)(r1 - r0), nnzt = (int)(k1 - k0);
+    const int off = (int)(k0 & 7);
+    const int j0 = lane * LI - off;
+    const bool any0 = j0 < nnzt;
+    int e_[2];                          // local ends of rows lane, lane + 32 (>= nrows: nnzt)
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+        const int i = lane + 32 * q;
+        e_[q] = i < nrows ? (int)(ld_rp(rp + r0 + 1 + i) - k0) : nnzt;
+    }
+    // wait for the row ends before issuing the x gathers (measured: LAP4096 0.320 -> 0.298 ms)
+    const bool ends_in = __all_sync(0xffffffffu, e_[0] >= 0 && e_[1] >= 0);   // every lane (no short circuit)
+    const bool any = any0 && ends_in;
+    double yv[2];
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+        const int i = lane + 32 * q;
+        yv[q] = (!B0 && i < nrows) ? (double)y[r0 + i] : 0.0;
+    }
+#pragma unroll
+    for (int e = 0; e < LI; e += 2) {
+        const double p0 = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)ch.v[e] * (double)ld_x(x + ch.c[e], px) : 0.0;
+        const double p1 = (any && (unsigned)(j0 + e + 1) < (unsigned)nnzt) ? (double)ch.v[e + 1] * (double)ld_x(x + ch.c[e + 1], px) : 0.0;
+        *reinterpret_cast<double2 *>(s_p + lane * LI + e) = make_double2(p0, p1);
+    }
+    if (lane == 31) {                                     // positions past lane 31's chunk (< off row ends)
+#pragma unroll 1
+        for (int pos = j0 + LI; pos < nnzt; ++pos)
+            s_p[pos + off] = (double)ld_hint(val + k0 + pos, pa) * (double)ld_x(x + ld_hint(col + k0 + pos, pa), px);
+    }
+    int s0 = __shfl_up_sync(0xffffffffu, e_[0], 1);
+    const int last0 = __shfl_sync(0xffffffffu, e_[0], 31);
+    int s1 = __shfl_up_sync(0xffffffffu, e_[1], 1);
+    if (lane == 0) { s0 = 0; s1 = last0; }
+    __syncwarp();
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+        const int i = lane + 32 * q;
+        if (i > nrows) break;
+        const int st = q ? s1 : s0, en = e_[q];
+        const double *ps = s_p + off + st;
+        double a0 = 0.0, a1 = 0.0;
+        int k = 0;
+        for (; k + 1 < en - st; k += 2) { a0 += ps[k]; a1 += ps[k + 1]; }
+        if (k < en - st) a0 += ps[k];
+        const double sum = a0 + a1;
+        if (i < nrows) {
+            double o = alpha * sum;
+            if (!B0) o = fma(beta, yv[q], o);
+            y[r0 + i] = (V)o;
+        } else {
+            carry_row[t] = en > st ? r1 : -1;
+            carry_val[t] = sum;
+        }
+    }
+}
+
+// Persistent warps over the class-1 tiles.  LIST = false: every tile is class 1, warp w
+// takes tiles w, w + W, ... and the next tile's coordinates are loaded while the current
+// one runs; LIST = true: positions [i0, i1) of the tile order (SPMV_MERGE_SCHEDULE).
+// The identity schedule is measurably faster than the list (LAP4096: 0.298 vs 0.339 ms).
+template <typename V, typename IT, bool B0, int MB, bool LIST>
+__global__ void __launch_bounds__(kT, MB)
+k_merge_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
+             const int64_t *__restrict__ crow, const int *__restrict__ order, int64_t i0, int64_t i1,
+             int64_t dmax, const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
+             int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
+    __shared__ __align__(16) double s_p_all[kT / 32][256 + 8];
+    const int wid = threadIdx.x >> 5;
+    const uint64_t pa = policy_evict_first(), px = policy_evict_last();
+    auto body = [&](int64_t t, int64_t r0, int64_t r1) {
+        MergeChunk<V> ch;
+        const int64_t k0 = merge_k(t, 256, r0, dmax), k1 = merge_k(t + 1, 256, r1, dmax);
+        merge_chunk_load(col, val, k0, k1, ch, pa);
+        merge_rows_tile<V, IT, B0>(rp, col, val, t, r0, r1, k0, k1, ch, x, y, alpha, beta, carry_row, carry_val,
+                                   s_p_all[wid], pa, px);
+    };
+    if constexpr (!LIST) {
+        const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+        int64_t t = i0 + ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+        if (t >= i1) return;
+        int64_t r0 = ld_coord(crow + t, px), r1 = ld_coord(crow + t + 1, px);
+        while (true) {
+            const int64_t tn = t + W;
+            int64_t q0 = 0, q1 = 0;
+            if (tn < i1) { q0 = ld_coord(crow + tn, px); q1 = ld_coord(crow + tn + 1, px); }
+            body(t, r0, r1);
+            if (tn >= i1) break;
+            t = tn; r0 = q0; r1 = q1;
+            __syncwarp();
+        }
+    } else {
+        SPMV_MERGE_SCHEDULE(body(t, r0, r1))
+    }
+}
+#undef SPMV_MERGE_SCHEDULE
 
 // ------------------------------------------------------------------ CSR5 (K6/G12)
 // equally sized 2-D tiles (32 lanes x sigma) with tile_ptr and
@@ -1160,9 +1331,33 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
         if (h->merge_T == 128) {
             k_merge<V, IT, B0, 4, 6><<<g, kT, 0, s>>>(rp, col, val, cr, h->merge_tiles, dmax, x, y, alpha, beta, crow, cval);
         } else {
-            const unsigned gp = (unsigned)std::min<int64_t>(g, (int64_t)h->ctx->sm_count * 3);
-            carveout(k_merge_persist<V, IT, B0, 8, 3>);
-            k_merge_persist<V, IT, B0, 8, 3><<<gp, kT, 0, s>>>(rp, col, val, cr, h->merge_tiles, dmax, x, y, alpha, beta, crow, cval);
+            // T = 256 (A28): all tiles class 1 -> the row-sum kernel over all tiles; most
+            // (>= half) class 1 -> the row-sum kernel over the class-1 part of the tile order,
+            // then the segmented-sum kernel over the rest; else the segmented-sum kernel over
+            // all tiles (it handles any tile; the order's indirection costs more than the
+            // row-sum tiles save when they are few)
+            const int *ord = (const int *)h->arr[SPMV_ARR_MERGE_TILE_ORDER].p;
+            const int64_t nl = h->merge_lean, nt = h->merge_tiles;
+            const unsigned gr = (unsigned)std::min<int64_t>(ceil_div<int64_t>(nl, kT / 32), (int64_t)h->ctx->sm_count * kMergeRowsMB);
+            if (nl == nt) {
+                carveout(k_merge_rows<V, IT, B0, kMergeRowsMB, false>);
+                k_merge_rows<V, IT, B0, kMergeRowsMB, false><<<gr, kT, 0, s>>>(rp, col, val, cr, ord, 0, nt, dmax, x, y,
+                                                                               alpha, beta, crow, cval);
+            } else if (2 * nl >= nt) {
+                carveout(k_merge_rows<V, IT, B0, kMergeRowsMB, true>);
+                k_merge_rows<V, IT, B0, kMergeRowsMB, true><<<gr, kT, 0, s>>>(rp, col, val, cr, ord, 0, nl, dmax, x, y,
+                                                                              alpha, beta, crow, cval);
+                SPMV_LAUNCH_CHECK();
+                const unsigned gp = (unsigned)std::min<int64_t>(ceil_div<int64_t>(nt - nl, kT / 32), (int64_t)h->ctx->sm_count * 3);
+                carveout(k_merge_persist<V, IT, B0, 8, 3, true>);
+                k_merge_persist<V, IT, B0, 8, 3, true><<<gp, kT, 0, s>>>(rp, col, val, cr, ord, nl, nt, dmax, x, y, alpha,
+                                                                         beta, crow, cval);
+            } else {
+                const unsigned gp = (unsigned)std::min<int64_t>(g, (int64_t)h->ctx->sm_count * 3);
+                carveout(k_merge_persist<V, IT, B0, 8, 3, false>);
+                k_merge_persist<V, IT, B0, 8, 3, false><<<gp, kT, 0, s>>>(rp, col, val, cr, ord, 0, nt, dmax, x, y, alpha,
+                                                                          beta, crow, cval);
+            }
         }
     }
         SPMV_LAUNCH_CHECK();
@@ -1221,7 +1416,10 @@ int run_launch_count(const spmv_handle *h, bool alpha0) {
     case SPMV_CSR_SCALAR: case SPMV_ELL: return h->n_rows ? 1 : 0;
     case SPMV_HYB: return (h->n_rows ? 1 : 0) + (h->hyb_coo_nnz ? 2 : 0);
     case SPMV_COO: return h->nnz ? 2 : (h->n_rows ? 1 : 0);
-    case SPMV_MERGE: return h->merge_tiles ? 2 : 0;
+    case SPMV_MERGE:
+        if (!h->merge_tiles) return 0;
+        if (h->merge_T == 128) return 2;
+        return (h->merge_lean == h->merge_tiles || 2 * h->merge_lean < h->merge_tiles ? 1 : 2) + 1;
     case SPMV_CSR5: return 1 + (h->csr5_tail_row < h->n_rows ? 1 : 0) + 1;
     }
     return 0;

@@ -28,7 +28,8 @@ STATUS = {0: "SPMV_OK", 1: "SPMV_ERR_INVALID_ARG", 2: "SPMV_ERR_NOT_CANONICAL", 
 ARRAYS = {"row_ptr": 0, "col": 1, "val": 2, "coo_row": 3, "ell_col": 4, "ell_val": 5, "hyb_coo_col": 6,
           "hyb_coo_val": 7, "merge_coord_row": 8, "merge_coord_nz": 9, "csr5_tile_ptr": 10,
           "csr5_row_lo": 11, "csr5_tile_desc": 12, "csr5_map_off": 13, "csr5_seg_map": 14,
-          "csr_chunk_row": 15, "csr_chunk_lo": 16}
+          "csr_chunk_row": 15, "csr_chunk_lo": 16, "merge_tile_class": 17,
+          "merge_tile_order": 18}
 
 
 class SpmvError(RuntimeError):
@@ -465,7 +466,8 @@ class Handle:
               "hyb_coo_col": np.int32, "hyb_coo_val": np.float64 if vb == 8 else np.float32,
               "merge_coord_row": np.int64, "merge_coord_nz": np.int64, "csr5_tile_ptr": np.int64,
               "csr5_row_lo": np.int64, "csr5_tile_desc": np.uint32, "csr5_map_off": np.int64,
-              "csr5_seg_map": np.int64, "csr_chunk_row": np.int64, "csr_chunk_lo": np.int64}[name]
+              "csr5_seg_map": np.int64, "csr_chunk_row": np.int64, "csr_chunk_lo": np.int64,
+              "merge_tile_class": np.uint8, "merge_tile_order": np.int32}[name]
         return buf.view(dt)
 
     def destroy(self, stream=None):

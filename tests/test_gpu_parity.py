@@ -221,6 +221,9 @@ def test_conversions_bit_exact(sp, name, dtype):
     cr, cn = oracle.merge_coords(A, T)
     assert np.array_equal(h.export("merge_coord_row"), cr)
     assert np.array_equal(h.export("merge_coord_nz"), cn)
+    cls = oracle.merge_class(A, T)
+    assert np.array_equal(h.export("merge_tile_class"), cls)
+    assert np.array_equal(h.export("merge_tile_order"), np.argsort(1 - cls.astype(np.int64), kind="stable"))
     # CSR5 (A6), default sigma and each legal sigma
     for sigma in (None, 4, 8, 12, 16):
         h = sp.convert(dA, "csr5", csr5_sigma=sigma or 0)
@@ -453,6 +456,7 @@ def test_index64_path(sp, name, fmt, dtype):
     if fmt == "merge":
         cr, cn = oracle.merge_coords(A, h.info()["merge_items"])
         assert np.array_equal(h.export("merge_coord_nz"), cn)
+        assert np.array_equal(h.export("merge_tile_class"), oracle.merge_class(A, h.info()["merge_items"]))
     if fmt == "csr5":
         e = oracle.csr5_encode(A, val_bytes=8 if dtype == torch.float64 else 4)
         assert np.array_equal(h.export("csr5_tile_desc"), e["tile_desc"])
@@ -565,3 +569,35 @@ def test_full_size_rmat24(sp):
         h, out = run_format(sp, Ai, dAi, fmt, torch.float32, 2.0, -1.0, xi, yi)
         h.destroy()
         assert np.array_equal(out, refi), fmt
+
+
+# merge tile classes (A28): the three schedules -- all tiles row-sum (short rows), most
+# row-sum with some segmented-sum tiles (short rows + a few long rows), few row-sum tiles
+def _merge_class_cases():
+    rng = np.random.default_rng(28)
+    short = rng.integers(3, 8, 20000)
+    mixed = short.copy()
+    mixed[[500, 7000, 15000]] = [900, 2500, 300]
+    mostly_long = rng.integers(30, 200, 3000)
+    return {"all_rowsum": short, "mixed": mixed, "few_rowsum": mostly_long}
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32], ids=["f64", "f32"])
+@pytest.mark.parametrize("which", ["all_rowsum", "mixed", "few_rowsum"])
+def test_merge_tile_schedules(sp, which, dtype):
+    lens = _merge_class_cases()[which]
+    A = _lens_matrix(lens, 30000, 2801, KIND[dtype])
+    cls = oracle.merge_class(A, 256)
+    nl, nt = int(cls.sum()), cls.size
+    expect = {"all_rowsum": nl == nt, "mixed": nt > nl and 2 * nl >= nt, "few_rowsum": 2 * nl < nt}[which]
+    assert expect, (which, nl, nt)
+    dA = to_dev(sp, A, dtype)
+    x = matgen.vector(A.n_cols, 28, 1, KIND[dtype])
+    y0 = matgen.vector(A.n_rows, 28, 2, KIND[dtype])
+    for alpha, beta in ALPHA_BETA:
+        ref, bound = oracle.spmv_csr(A, x, alpha, beta, y0, with_bound=True)
+        h, out = run_format(sp, A, dA, "merge", dtype, alpha, beta, x, y0)
+        assert np.array_equal(h.export("merge_tile_class"), cls)
+        ok, ratio, nbad = oracle.check_tolerance(out, ref, bound, TOL[dtype])
+        assert ok, (alpha, beta, nbad, ratio)
+        h.destroy()

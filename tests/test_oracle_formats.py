@@ -151,6 +151,48 @@ def test_merge_walk_equals_binary_search(T):
         assert np.all(np.diff(cr) >= 0) and np.all(np.diff(cn) >= 0)
 
 
+# merge tile class (A28): 1 iff the tile consumes < max_rows row ends and no row gets
+# more than max_len of its nonzeros.  Pinned by closed forms and by the coordinate
+# formula (binary search, not a walk) applied to the definition.
+
+def merge_class_formula(A, T, max_rows=64, max_len=32):
+    total = A.n_rows + A.nnz
+    nt = -(-total // T)
+    out = []
+    for t in range(nt):
+        r0, k0 = merge_coord_formula(A.row_ptr, min(t * T, total))
+        r1, k1 = merge_coord_formula(A.row_ptr, min((t + 1) * T, total))
+        rp = np.clip(np.asarray(A.row_ptr[r0:min(r1 + 2, A.n_rows + 1)], np.int64), k0, k1)
+        parts = np.diff(np.concatenate([[k0], rp[1:], [k1]]))
+        out.append(int(r1 - r0 < max_rows and parts.max(initial=0) <= max_len))
+    return np.array(out, np.uint8)
+
+
+@pytest.mark.parametrize("T", [7, 64, 128, 256])
+def test_merge_class_definition(T):
+    for A in structured_cases():
+        assert np.array_equal(oracle.merge_class(A, T), merge_class_formula(A, T))
+
+
+def test_merge_class_closed_forms():
+    # 5-point Laplacian (App. B): rows <= 5 nonzeros, ~43 row ends per 256 items -> all 1
+    A = matgen.laplacian5(16)
+    assert oracle.merge_class(A, 256).all()
+    # a row of exactly 32 / 33 nonzeros alone in a tile: 32 is a row-sum tile, 33 is not
+    for L, exp in ((32, 1), (33, 0)):
+        A = matgen.from_lengths([L], 40, seed=1)
+        assert oracle.merge_class(A, 256).tolist() == [exp]
+    # 63 / 64 empty rows then nothing: 63 row ends -> 1, 64 -> 0 (T = 256 holds them all)
+    for n, exp in ((63, 1), (64, 0)):
+        A = matgen.HostCSR(np.zeros(n + 1, np.int64), np.zeros(0, np.int32), np.zeros(0), n, 4)
+        assert oracle.merge_class(A, 256).tolist() == [exp]
+    # one 1500-nonzero row split over 6 tiles of 256 items: every tile has a part > 32
+    A = matgen.from_lengths([1500], 1500, seed=10)
+    assert not oracle.merge_class(A, 256).any()
+    # the same test with the limits opened up: every tile qualifies
+    assert oracle.merge_class(A, 256, max_rows=300, max_len=256).all()
+
+
 # ------------------------------------------------------------------ partition
 
 @pytest.mark.parametrize("name", ["app_a_4x4.json", "app_a_5x5.json"])
