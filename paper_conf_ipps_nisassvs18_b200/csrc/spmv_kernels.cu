@@ -29,7 +29,8 @@ constexpr int kIPT = kItemsPerThread;
 constexpr int kWIPT = kWarpItemsPerLane;
 constexpr int kMinBlocks = 4;   // 4 CTAs x 256 threads per SM: <= 64 registers
 constexpr int kFold = 256;
-constexpr int kMergeRowsMB = 4;   // k_merge_rows CTAs per SM   // sequential steps per accumulator before folding (A13)
+constexpr int kMergeRowsMB = 4;   // k_merge_rows CTAs per SM
+constexpr int kCsrRowsMB = 4;     // k_csr_rows CTAs per SM   // sequential steps per accumulator before folding (A13)
 
 // ------------------------------------------------------------------ helpers
 
@@ -550,6 +551,122 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
                 if (!B0) o = fma(beta, yv[q], o);
                 y[Wlo + i] = (V)o;
             }
+        }
+    }
+}
+
+// ------------------------------------------------------------------ CSR row batches (A29)
+// Short rows (vector width W <= 8, A5): a warp takes 32 consecutive rows, whose nonzeros
+// [rp[b], rp[b+32]) are contiguous -- lane l loads the 32-byte aligned chunk of 8
+// nonzeros starting at (rp[b] rounded down to 8) + 8l with 256-bit loads, the products
+// go to shared memory in that order and lane i sums row b + i sequentially (<= 32
+// terms, two accumulators).  The batch's row pointers arrive one batch ahead.  A batch
+// whose rows do not fit (a row > 32 nonzeros, or > 256 - (rp[b] mod 8) nonzeros in
+// all) is reduced row by row by the whole warp (the paper's warp-per-row vector
+// kernel; blocked summation, A13).  CHUNKED: rows longer than long_len
+// get beta*y here and their chunks arrive through the fix-up (A25).
+template <typename V, typename IT, bool B0, int MB, bool CHUNKED>
+__global__ void __launch_bounds__(kT, MB)
+k_csr_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
+           const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta, int64_t long_len) {
+    __shared__ __align__(16) double s_p_all[kT / 32][256 + 8];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    double *s_p = s_p_all[wid];
+    const int64_t gwarp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const uint64_t pa = policy_evict_first(), px = policy_evict_last();
+    int64_t b = gwarp * 32;
+    IT nlo = 0, nhi = 0;                          // row pointers of the next batch (prefetched)
+    if (b < n) {
+        nlo = __ldg(rp + (b + lane < n ? b + lane : n));
+        nhi = __ldg(rp + (b + 32 < n ? b + 32 : n));
+    }
+    for (; b < n; b += nwarps * 32) {
+        const int64_t my_a = (int64_t)nlo;
+        const int64_t hi = (int64_t)nhi;
+        const int64_t nb = b + nwarps * 32;
+        if (nb < n) {
+            nlo = __ldg(rp + (nb + lane < n ? nb + lane : n));
+            nhi = __ldg(rp + (nb + 32 < n ? nb + 32 : n));
+        }
+        const int64_t lo = __shfl_sync(0xffffffffu, my_a, 0);
+        const int64_t nx = __shfl_down_sync(0xffffffffu, my_a, 1);
+        const int64_t my_e = lane == 31 ? hi : nx;    // rows >= n: my_a = my_e = rp[n]
+        const bool in_row = b + lane < n;
+        const double yv = (!B0 && in_row) ? (double)y[b + lane] : 0.0;
+        const int off = (int)(lo & 7);
+        const int cnt = (int)(hi - lo < (1 << 20) ? hi - lo : (1 << 20));
+        double sum = 0.0;
+        if (__all_sync(0xffffffffu, my_e - my_a <= 32) && cnt + off <= 256) {
+            const int j0 = lane * 8 - off;
+            const int64_t base = lo - off + lane * 8;
+            double p[8];
+            if (j0 < cnt) {
+                int c[8];
+                V v[8];
+                ld256(col + base, c, pa);
+                if constexpr (sizeof(V) == 8) {          // second sector only if it holds a batch element
+                    double a4[4], b4[4];
+                    ld256(reinterpret_cast<const double *>(val + base), a4, pa);
+                    if (j0 + 4 < cnt) ld256(reinterpret_cast<const double *>(val + base + 4), b4, pa);
+                    else { b4[0] = b4[1] = b4[2] = b4[3] = 0.0; }
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) { v[q] = (V)a4[q]; v[4 + q] = (V)b4[q]; }
+                } else {
+                    VecLoad8<V>::load(val + base, v, pa);
+                }
+#pragma unroll
+                for (int e = 0; e < 8; ++e)
+                    p[e] = (unsigned)(j0 + e) < (unsigned)cnt ? (double)v[e] * (double)ld_x(x + c[e], px) : 0.0;
+            } else {
+#pragma unroll
+                for (int e = 0; e < 8; ++e) p[e] = 0.0;
+            }
+#pragma unroll
+            for (int e = 0; e < 8; e += 2) *reinterpret_cast<double2 *>(s_p + lane * 8 + e) = make_double2(p[e], p[e + 1]);
+            __syncwarp();
+            const int st = (int)(my_a - lo);
+            int len = (int)(my_e - my_a);
+            if (CHUNKED && len > long_len) len = 0;            // A25: chunks via the fix-up
+            const double *ps = s_p + off + st;
+            double a0 = 0.0, a1 = 0.0;
+            int k = 0;
+            for (; k + 1 < len; k += 2) { a0 += ps[k]; a1 += ps[k + 1]; }
+            if (k < len) a0 += ps[k];
+            sum = a0 + a1;
+            __syncwarp();
+        } else {
+            // row by row, the whole warp on each (8 loads per lane in flight)
+            for (int i = 0; i < 32; ++i) {
+                const int64_t ra = __shfl_sync(0xffffffffu, my_a, i), rb = __shfl_sync(0xffffffffu, my_e, i);
+                if (CHUNKED && rb - ra > long_len) continue;   // A25: chunks via the fix-up
+                double tot = 0.0, acc[8];
+#pragma unroll
+                for (int q = 0; q < 8; ++q) acc[q] = 0.0;
+                int it = 0;
+                int64_t k = ra + lane;
+                for (; k + 7 * 32 < rb; k += 8 * 32) {
+                    int d[8];
+                    V w[8];
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(x + d[q], px);
+                    if (++it == kFold) {
+#pragma unroll
+                        for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
+                        it = 0;
+                    }
+                }
+                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
+                const double part = warp_sum(tot + (((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]))));
+                if (lane == i) sum = part;
+            }
+        }
+        if (in_row) {
+            double o = alpha * sum;
+            if (!B0) o = fma(beta, yv, o);
+            y[b + lane] = (V)o;
         }
     }
 }
@@ -1249,6 +1366,17 @@ spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col
                               int64_t n, int w, double alpha, double beta, cudaStream_t s,
                               int64_t long_len = INT64_MAX) {
     if (n == 0) return SPMV_OK;
+    // W <= 8: 32-row batches (A29) when col/val are 32-byte aligned (the chunk loads)
+    static const bool rows_on = [] { const char *e = getenv("SPMV_CSR_ROWS"); return !e || atoi(e) != 0; }();
+    if (w <= 8 && rows_on && ((((uintptr_t)col) | ((uintptr_t)val)) & 31) == 0) {
+        const unsigned gr = (unsigned)std::min<int64_t>(ceil_div<int64_t>(n, kT), (int64_t)h->ctx->sm_count * kCsrRowsMB);
+        if (long_len == INT64_MAX)
+            k_csr_rows<V, IT, B0, kCsrRowsMB, false><<<gr, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len);
+        else
+            k_csr_rows<V, IT, B0, kCsrRowsMB, true><<<gr, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len);
+        SPMV_LAUNCH_CHECK();
+        return SPMV_OK;
+    }
     // 16 CTAs (4096 threads) per SM of grid-stride warps
     const int64_t threads = ceil_div<int64_t>(n, 32 / w) * 32;
     const int g = grid_stride_blocks(h->ctx, threads, 16);
