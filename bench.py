@@ -53,6 +53,12 @@ def build_matrix(name, dtype_kind):
         return matgen.laplacian5(int(name[3:]))
     if name.startswith("rmat"):
         return matgen.rmat(int(name[4:]), kind=dtype_kind)
+    if name.startswith("mtx:"):                     # a Matrix Market file
+        from matgen.mtx import read_mtx
+        A = read_mtx(name[4:])
+        if dtype_kind == "f32":
+            A.val = A.val.astype("float32").astype("float64")
+        return A
     raise SystemExit(f"unknown config {name}")
 
 

@@ -580,6 +580,29 @@ __device__ __forceinline__ double row_walk(const int *s_c, const V *s_v, int st,
     }
     return a0 + a1;
 }
+// the same walk reading col/val from global memory (rows of a batch that does not fit
+// the shared-memory chunk)
+template <typename V>
+__device__ __forceinline__ double row_walk_global(const int *__restrict__ col, const V *__restrict__ val, int64_t a,
+                                                  int len, const V *__restrict__ x, uint64_t pa, uint64_t px) {
+    double a0 = 0.0, a1 = 0.0;
+    for (int k = 0; k < len; k += 8) {
+        int cc[8];
+        V vv[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+            const bool in = k + u < len;
+            cc[u] = in ? ld_hint(col + a + k + u, pa) : 0;
+            vv[u] = in ? ld_hint(val + a + k + u, pa) : (V)0;
+        }
+        double pp[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) pp[u] = k + u < len ? (double)vv[u] * (double)ld_x(x + cc[u], px) : 0.0;
+#pragma unroll
+        for (int u = 0; u < 8; u += 2) { a0 += pp[u]; a1 += pp[u + 1]; }
+    }
+    return a0 + a1;
+}
 // a lane's 8-element chunk into shared memory (16-byte stores)
 template <typename V>
 __device__ __forceinline__ void chunk_store(int *s_c, V *s_v, int pos, const int (&c)[8], const V (&v)[8]) {
@@ -664,10 +687,17 @@ k_csr_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
             sum = row_walk(s_c, s_v, (int)(my_a - lo) + off, len, x, px);
             __syncwarp();
         } else {
-            // row by row, the whole warp on each (8 loads per lane in flight)
-            for (int i = 0; i < 32; ++i) {
+            // rows <= 32 nonzeros: lane i walks row b + i straight from global memory;
+            // longer rows: the whole warp on each (8 loads per lane in flight)
+            int64_t len = my_e - my_a;
+            if (CHUNKED && len > long_len) len = 0;            // A25: chunks via the fix-up
+            const bool lng = len > 32;
+            if (!lng) sum = row_walk_global(col, val, my_a, (int)len, x, pa, px);
+            unsigned lm = __ballot_sync(0xffffffffu, lng);
+            while (lm) {
+                const int i = __ffs(lm) - 1;
+                lm &= lm - 1;
                 const int64_t ra = __shfl_sync(0xffffffffu, my_a, i), rb = __shfl_sync(0xffffffffu, my_e, i);
-                if (CHUNKED && rb - ra > long_len) continue;   // A25: chunks via the fix-up
                 double tot = 0.0, acc[8];
 #pragma unroll
                 for (int q = 0; q < 8; ++q) acc[q] = 0.0;

@@ -26,17 +26,50 @@ LABEL_SETS = {
     "label6": ("coo", "ell", "csr", "hyb", "merge", "csr5"),
     "label5": ("ell", "csr", "hyb", "merge", "csr5"),
     "label3": ("ell", "csr", "hyb"),
+    # the scalar CSR kernel ("a thread to process each
+    # row") as a seventh class; emitted only when it was timed
+    "label7": ("coo", "ell", "csr", "hyb", "merge", "csr5", "csr_scalar"),
 }
+LABEL_ORDER = PAPER_FORMATS + ("csr_scalar",)   # exact ties: Fig. 3 order, then the variant
+
+
+class L2Flush:
+    """Cold-L2 timing (A11 variant): writing a buffer of twice the L2
+    size between runs evicts A, x and y.  Measurement plumbing, not the hot path."""
+
+    def __init__(self, device=None):
+        props = torch.cuda.get_device_properties(device or torch.cuda.current_device())
+        self.buf = torch.empty(2 * int(props.L2_cache_size), dtype=torch.uint8,
+                               device=device or torch.cuda.current_device())
+        self.n = 0
+
+    def __call__(self):
+        self.n += 1
+        self.buf.fill_(self.n & 0xFF)
 
 
 def time_handle(h, x: torch.Tensor, y: torch.Tensor, reps: int = 50, warmup: int = 5,
-                alpha: float = 1.0, beta: float = 1.0, per_call: bool = True) -> Dict[str, float]:
+                alpha: float = 1.0, beta: float = 1.0, per_call: bool = True,
+                flush: Optional[L2Flush] = None) -> Dict[str, float]:
     """A11 protocol on the current stream.  Returns mean (batch event pair), median and
-    min of per-call events, in milliseconds."""
+    min of per-call events, in milliseconds.  With `flush` (cold L2): every run is
+    preceded by an L2 flush outside its event pair; mean/median/min are over the
+    per-call events."""
     s = torch.cuda.current_stream()
     for _ in range(warmup):
         h.run(alpha, x, beta, y)
     s.synchronize()
+    if flush is not None:
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+        for a, b in evs:
+            flush()
+            a.record(s)
+            h.run(alpha, x, beta, y)
+            b.record(s)
+        s.synchronize()
+        ts = [a.elapsed_time(b) for a, b in evs]
+        return {"t_mean_ms": sum(ts) / len(ts), "t_median_ms": statistics.median(ts), "t_min_ms": min(ts),
+                "reps": reps, "cold_l2": True}
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     t0.record(s)
     for _ in range(reps):
@@ -61,7 +94,9 @@ def labels(times_ms: Dict[str, Optional[float]]) -> Dict[str, object]:
     """A12: argmin over feasible formats per label set; exact ties in Fig. 3 order."""
     out: Dict[str, object] = {}
     for name, fmts in LABEL_SETS.items():
-        feas = [(times_ms[f], PAPER_FORMATS.index(f), f) for f in fmts if times_ms.get(f) is not None]
+        if name == "label7" and "csr_scalar" not in times_ms:
+            continue
+        feas = [(times_ms[f], LABEL_ORDER.index(f), f) for f in fmts if times_ms.get(f) is not None]
         if not feas:
             out[name] = None
             continue
@@ -74,7 +109,7 @@ def labels(times_ms: Dict[str, Optional[float]]) -> Dict[str, object]:
 
 def measure_matrix(A: CSR, formats: Iterable[str] = PAPER_FORMATS, reps: int = 50, warmup: int = 5,
                    x: Optional[torch.Tensor] = None, y: Optional[torch.Tensor] = None,
-                   **convert_opts) -> Dict[str, object]:
+                   cold_l2: bool = False, **convert_opts) -> Dict[str, object]:
     """Convert A to each format, time it, and emit the per-format record + labels
     (the paper's ground truth, regenerated on this GPU).  Before timing, every format's
     y = A x + y0 is compared with the CSR result (max |diff| / (max |y| + 1) recorded
@@ -86,6 +121,8 @@ def measure_matrix(A: CSR, formats: Iterable[str] = PAPER_FORMATS, reps: int = 5
         y = torch.zeros(A.n_rows, dtype=A.dtype, device=dev)
     rec: Dict[str, object] = {"formats": {}}
     times: Dict[str, Optional[float]] = {}
+    cold: Dict[str, Optional[float]] = {}
+    flush = L2Flush(dev) if cold_l2 else None
     ref_y = None
     for f in formats:
         try:
@@ -94,6 +131,7 @@ def measure_matrix(A: CSR, formats: Iterable[str] = PAPER_FORMATS, reps: int = 5
             if e.status in (3, 4):          # SPMV_ERR_SIZE / NO_MEMORY -> N/A (A4)
                 rec["formats"][f] = {"status": "N/A", "reason": e.name}
                 times[f] = None
+                cold[f] = None
                 continue
             raise
         yc = y.clone()
@@ -108,13 +146,20 @@ def measure_matrix(A: CSR, formats: Iterable[str] = PAPER_FORMATS, reps: int = 5
         rec["formats"][f] = {**t, "gflops": gflops, "gbs_own": gbs, "bytes_per_run": info["bytes_per_run"],
                              "launches": h.launches(), "agree": agree}
         times[f] = t["t_mean_ms"]
+        if flush is not None:
+            tc = time_handle(h, x, y.clone(), reps=reps, warmup=warmup, flush=flush)
+            rec["formats"][f]["cold"] = tc
+            cold[f] = tc["t_mean_ms"]
         h.destroy()
     rec.update(labels(times))
+    if flush is not None:
+        rec["cold_labels"] = labels(cold)
     return rec
 
 
 def sweep(start: int = 0, count: int = 2000, out: str = "sweep.jsonl", dtype: str = "f64", reps: int = 50,
-          warmup: int = 5, shard: int = 0, nshards: int = 1, max_nnz: Optional[int] = None) -> int:
+          warmup: int = 5, shard: int = 0, nshards: int = 1, max_nnz: Optional[int] = None,
+          cold_l2: bool = False, with_scalar: bool = False) -> int:
     """BASELINE configs[3]: the format-selection sweep.  Matrices start..start+count-1
     (matgen.sweep_matrix, seeded), this process takes i % nshards == shard (replicas over
     GPUs).  One JSONL record per matrix: generator parameters, the 17 features + extras
@@ -148,7 +193,8 @@ def sweep(start: int = 0, count: int = 2000, out: str = "sweep.jsonl", dtype: st
             feats = features(dA)
             x = torch.from_numpy(matgen.vector(A.n_cols, p["seed"], 1, dtype)).to(dA.row_ptr.device).to(tdt)
             y = torch.from_numpy(matgen.vector(A.n_rows, p["seed"], 2, dtype)).to(dA.row_ptr.device).to(tdt)
-            rec = measure_matrix(dA, reps=reps, warmup=warmup, x=x, y=y)
+            fmts = PAPER_FORMATS + (("csr_scalar",) if with_scalar else ())
+            rec = measure_matrix(dA, formats=fmts, reps=reps, warmup=warmup, x=x, y=y, cold_l2=cold_l2)
             row = {"i": i, "params": p, "dtype": dtype, "n_rows": A.n_rows, "n_cols": A.n_cols, "nnz": A.nnz,
                    "features": {k: feats[k] for k in PAPER_FEATURES},
                    "extras": {k: feats[k] for k in ("ell_width", "ell_slots", "ell_pad_frac", "hyb_width",
@@ -182,13 +228,15 @@ def _main():
     ap.add_argument("--reps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--max-nnz", type=int, default=None)
+    ap.add_argument("--cold-l2", action="store_true", help="also time every format with L2 flushed before each run")
+    ap.add_argument("--with-scalar", action="store_true", help="time CSR-scalar too and emit label7")
     a = ap.parse_args()
     import os
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
     out = a.out if ws == 1 else a.out.replace(".jsonl", f".rank{rank}.jsonl")
-    n = sweep(a.start, a.count, out, a.dtype, a.reps, a.warmup, rank, ws, a.max_nnz)
+    n = sweep(a.start, a.count, out, a.dtype, a.reps, a.warmup, rank, ws, a.max_nnz, a.cold_l2, a.with_scalar)
     print(f"rank {rank}: measured {n} matrices -> {out}")
 
 

@@ -601,3 +601,20 @@ def test_merge_tile_schedules(sp, which, dtype):
         ok, ratio, nbad = oracle.check_tolerance(out, ref, bound, TOL[dtype])
         assert ok, (alpha, beta, nbad, ratio)
         h.destroy()
+
+
+def test_harness_record_cold_l2_and_scalar(sp):
+    """The timing/label harness (a16) on one matrix: every format timed hot and cold
+    (L2 flushed before each run), labels over six and seven classes,
+    each format's y agreeing with CSR's."""
+    from paper_conf_ipps_nisassvs18_b200 import harness
+    A = _lens_matrix(np.random.default_rng(5).integers(0, 20, 3000), 3000, 55)
+    dA = to_dev(sp, A, torch.float64)
+    rec = harness.measure_matrix(dA, formats=sp.PAPER_FORMATS + ("csr_scalar",), reps=5, warmup=2, cold_l2=True)
+    assert rec["label6"] in sp.PAPER_FORMATS and rec["label7"] in sp.PAPER_FORMATS + ("csr_scalar",)
+    assert rec["cold_labels"]["label6"] in sp.PAPER_FORMATS
+    for f, r in rec["formats"].items():
+        if r.get("status") == "N/A":
+            continue
+        assert r["agree"] < 1e-12, f
+        assert r["cold"]["cold_l2"] and r["cold"]["t_mean_ms"] > 0 and r["t_mean_ms"] > 0

@@ -17,6 +17,16 @@ def test_label_rules():
     assert tie["label6"] == "ell" and tie["label3"] == "ell"
     none = labels({f: None for f in LABEL_SETS["label6"]})
     assert none["label6"] is None
+    assert "label7" not in lab                       # CSR-scalar not timed -> no label7
+
+
+def test_label7_scalar_class():
+    """CSR-scalar as a seventh class; ties go to the paper's six first."""
+    t = {"coo": 3.0, "ell": None, "csr": 2.0, "hyb": 2.5, "merge": 2.2, "csr5": 2.4, "csr_scalar": 1.5}
+    lab = labels(t)
+    assert lab["label7"] == "csr_scalar" and lab["label6"] == "csr"
+    lab = labels({**t, "csr_scalar": 2.0})
+    assert lab["label7"] == "csr"
 
 
 def test_sweep_recipe_deterministic_and_canonical():
