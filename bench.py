@@ -318,7 +318,20 @@ def run_ours(args):
     fmts = [f for f in formats if f in handles]
     ys = {f: y_init.clone() for f in fmts}
     split = {}
-    if ws > 1 and args.overlap:
+    halo = None
+    if ws > 1 and args.halo:
+        # halo exchange: each rank receives only the x entries its rows
+        # reference, point to point (all_to_all_single), own-column blocks overlap it
+        from paper_conf_ipps_nisassvs18_b200.dist import HaloPlan
+        from paper_conf_ipps_nisassvs18_b200.spmv import spmv_slice_split
+        lay = dsp.layout
+        halo = HaloPlan(dA.row_ptr, dA.col, A.n_cols, lay.splits, lay.rank)
+        split = {f: (sp.convert(spmv_slice_split(dA, lay.splits, lay.rank, 0), f),
+                     sp.convert(spmv_slice_split(dA, lay.splits, lay.rank, 1, halo.colmap, halo.S), f)) for f in fmts}
+        x_own = torch.from_numpy(x_h[lay.r0:lay.r1].copy()).cuda().to(dtype)
+        halo_send = torch.zeros(halo.send_index.numel(), dtype=dtype, device="cuda")
+        halo_recv = torch.zeros(halo.recv_len, dtype=dtype, device="cuda")
+    elif ws > 1 and args.overlap:
         split = {f: dsp.split_handles(f) for f in fmts}
         x_own = torch.from_numpy(x_h[dsp.layout.r0:dsp.layout.r1].copy()).cuda().to(dtype)
 
@@ -359,6 +372,16 @@ def run_ours(args):
         dist.barrier()
 
     def step(record=None):
+        if halo is not None:
+            from paper_conf_ipps_nisassvs18_b200.spmv import spmv_gather
+            spmv_gather(x_own, halo.send_index, halo_send)
+            work = halo.exchange(halo_send, halo_recv, async_op=True)
+            for f in fmts:
+                split[f][0].run(1.0, x_own, 1.0, ys[f])
+            work.wait()
+            for f in fmts:
+                split[f][1].run(1.0, halo_recv, 1.0, ys[f])
+            return
         if split:
             # overlap: own-column blocks while the all-gather is in flight
             work = dsp.exchange_async()
@@ -468,11 +491,14 @@ def run_ours(args):
                        "n_rows": A.n_rows, "n_cols": A.n_cols, "nnz": A.nnz, "formats": fmts,
                        "step": "one SpMV (alpha=1, beta=1) in each feasible format",
                        "l2": "no flush: every format's arrays exceed the 126 MB L2",
-                       "parallelism": (f"row-partitioned x{ws}, NCCL all-gather of x"
-                                       + (" (compressed)" if args.compress else "")
-                                       + (" overlapped with own-column blocks" if args.overlap else ""))
+                       "parallelism": ((f"row-partitioned x{ws}, NCCL all_to_all halo exchange of x overlapped "
+                                        "with own-column blocks") if halo is not None else
+                                       (f"row-partitioned x{ws}, NCCL all-gather of x"
+                                        + (" (compressed)" if args.compress else "")
+                                        + (" overlapped with own-column blocks" if args.overlap else "")))
                                       if ws > 1 else "1 GPU",
-                       "exchange_bytes_per_rank": dsp.exchange_bytes() if dsp is not None else 0},
+                       "exchange_bytes_per_rank": (halo.exchange_bytes(ys[fmts[0]].element_size()) if halo is not None
+                                                   else dsp.exchange_bytes() if dsp is not None else 0)},
             "per_format": per_format, "best_format": best,
             "roofline": roof(dom), "roofline_best": roof(best),
             "features": {"ms": feat_ms, "gbs": (4 * A.nnz + 8 * (A.n_rows + 1)) / (feat_ms * 1e-3) / 1e9,
@@ -510,6 +536,8 @@ def main():
     ap.add_argument("--formats", default="")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--compress", action="store_true", help="N > 1: exchange only referenced columns")
+    ap.add_argument("--halo", action="store_true",
+                    help="N > 1: point-to-point halo exchange of the referenced x entries (all_to_all_single)")
     ap.add_argument("--overlap", action="store_true",
                     help="N > 1: own-column blocks run while the x all-gather is in flight")
     ap.add_argument("--e2e-steps", type=int, default=10)

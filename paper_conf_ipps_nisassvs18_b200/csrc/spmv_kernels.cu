@@ -15,6 +15,7 @@
 #include <climits>
 #include <cstdlib>
 #include <cstring>
+#include <type_traits>
 
 #include "internal.h"
 #include "kernels.h"
@@ -603,6 +604,30 @@ __device__ __forceinline__ double row_walk_global(const int *__restrict__ col, c
     }
     return a0 + a1;
 }
+// positions [0, n) (n <= 256) of a 32-byte aligned global run into shared memory, in
+// warp-contiguous 16-byte pieces (lane l: piece l + 32q); pieces starting at or past n
+// are not read (a piece holding the last element stays inside that element's sector)
+template <typename T>
+__device__ __forceinline__ void stage_pieces(const T *__restrict__ g, T *s, int n, uint64_t pa) {
+    constexpr int E = 16 / sizeof(T);                    // elements per piece
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int q = 0; q < 256 / (32 * E); ++q) {
+        const int pos = (lane + 32 * q) * E;
+        if (pos < n) {
+            if constexpr (sizeof(T) == 8) {
+                const double2 w = ld_hint(reinterpret_cast<const double2 *>(g + pos), pa);
+                *reinterpret_cast<double2 *>(s + pos) = w;
+            } else if constexpr (std::is_same<T, float>::value) {
+                const float4 w = ld_hint(reinterpret_cast<const float4 *>(g + pos), pa);
+                *reinterpret_cast<float4 *>(s + pos) = w;
+            } else {
+                const int4 w = ld_hint(reinterpret_cast<const int4 *>(g + pos), pa);
+                *reinterpret_cast<int4 *>(s + pos) = w;
+            }
+        }
+    }
+}
 // a lane's 8-element chunk into shared memory (16-byte stores)
 template <typename V>
 __device__ __forceinline__ void chunk_store(int *s_c, V *s_v, int pos, const int (&c)[8], const V (&v)[8]) {
@@ -665,22 +690,12 @@ k_csr_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
             // products-to-shared variant, lane chunks gathering, was 0.312 vs 0.297 ms)
             int *s_c = reinterpret_cast<int *>(s_p + 264);
             V *s_v = reinterpret_cast<V *>(s_p);
-            if (j0 < cnt) {
-                int c[8];
-                V v[8];
-                ld256(col + base, c, pa);
-                if constexpr (sizeof(V) == 8) {          // second sector only if it holds a batch element
-                    double a4[4], b4[4];
-                    ld256(reinterpret_cast<const double *>(val + base), a4, pa);
-                    if (j0 + 4 < cnt) ld256(reinterpret_cast<const double *>(val + base + 4), b4, pa);
-                    else { b4[0] = b4[1] = b4[2] = b4[3] = 0.0; }
-#pragma unroll
-                    for (int q = 0; q < 4; ++q) { v[q] = (V)a4[q]; v[4 + q] = (V)b4[q]; }
-                } else {
-                    VecLoad8<V>::load(val + base, v, pa);
-                }
-                chunk_store(s_c, s_v, lane * 8, c, v);
-            }
+            // warp-contiguous 16-byte pieces: each load / store instruction covers 512
+            // consecutive bytes (no shared-memory bank conflicts; lane chunks of 32 / 64 B
+            // made the stores 2- / 4-way conflicted); pieces past the batch are skipped
+            stage_pieces(col + (lo - off), s_c, cnt + off, pa);
+            stage_pieces(val + (lo - off), s_v, cnt + off, pa);
+            (void)j0; (void)base;
             __syncwarp();
             int len = (int)(my_e - my_a);
             if (CHUNKED && len > long_len) len = 0;            // A25: chunks via the fix-up

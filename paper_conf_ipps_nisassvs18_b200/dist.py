@@ -197,3 +197,104 @@ class DistSpMV:
         all_gather_slots(buf, slot, self.group)
         return torch.cat([buf[k * S: k * S + int(self.layout.splits[k + 1] - self.layout.splits[k])]
                           for k in range(P)])
+
+
+# ---------------------------------------------------------------------- halo exchange
+
+class HaloPlan:
+    """Point-to-point halo exchange for a row partition: receiver k gets,
+    from each owner o != k, exactly the x entries of o's rows that k's rows reference,
+    padded to S_k = max_o (count from o).  Receiver k's buffer holds slot o at
+    [o*S_k, o*S_k + count); `colmap` maps each foreign column j referenced by this rank to
+    its buffer position (-1 elsewhere), the layout ``spmv_slice_split(which=1, colmap)``
+    remaps the foreign block through.  A banded matrix (LAP) exchanges its 2 x band
+    rows per rank instead of the whole x.  Built once with tensor index ops on the
+    matrix's device (setup plumbing); a step is one ``spmv_gather`` pack + one
+    all_to_all_single.  Pure index logic: the gloo tests run it on CPU tensors."""
+
+    def __init__(self, row_ptr: torch.Tensor, col: torch.Tensor, n_cols: int, splits, rank: int):
+        dev = col.device
+        sp = torch.as_tensor(np.asarray(splits, np.int64), device=dev)
+        P = int(sp.numel() - 1)
+        self.P, self.rank, self.splits = P, rank, np.asarray(splits, np.int64)
+        self.slots = []                  # S_k per receiver
+        send = []                        # this rank's pack indices, per receiver, padded to S_k
+        self.sent_counts = []
+        self.colmap = torch.full((n_cols,), -1, dtype=torch.int32, device=dev)
+        for k in range(P):
+            a, b = int(row_ptr[int(self.splits[k])]), int(row_ptr[int(self.splits[k + 1])])
+            cols = col[a:b].to(torch.int64)
+            own = torch.searchsorted(sp, cols, right=True) - 1
+            u = torch.unique(cols[own != k])                   # sorted foreign columns of k
+            ou = torch.searchsorted(sp, u, right=True) - 1
+            cnt = torch.bincount(ou, minlength=P) if u.numel() else torch.zeros(P, dtype=torch.int64, device=dev)
+            S = max(int(cnt.max()), 1)
+            self.slots.append(S)
+            first = torch.cumsum(cnt, 0) - cnt                 # start of each owner's run in u
+            pos = torch.arange(u.numel(), device=dev) - first[ou]
+            if k == rank:
+                self.colmap[u] = (ou * S + pos).to(torch.int32)
+            mine = u[ou == rank] - int(self.splits[rank])
+            self.sent_counts.append(int(mine.numel()))
+            pad = torch.zeros(S, dtype=torch.int32, device=dev)
+            pad[: mine.numel()] = mine.to(torch.int32)
+            send.append(pad)
+        self.send_index = torch.cat(send)                       # length sum_k S_k
+        self.S = self.slots[rank]                               # this rank's receive slot
+
+    @property
+    def recv_len(self) -> int:
+        return self.P * self.S
+
+    def exchange_bytes(self, elem: int) -> int:
+        """Bytes this rank receives per step (padded slots, self excluded)."""
+        return (self.P - 1) * self.S * elem
+
+    def exchange(self, send_buf: torch.Tensor, recv_buf: torch.Tensor, group=None, async_op: bool = False):
+        return dist.all_to_all_single(recv_buf, send_buf, output_split_sizes=[self.S] * self.P,
+                                      input_split_sizes=list(self.slots), group=group, async_op=async_op)
+
+
+class HaloSpMV:
+    """Row-partitioned y = alpha*A*x + beta*y with a halo exchange instead of the x
+    all-gather.  Own-column block on the rank's x slice (overlapping
+    the exchange on NCCL), foreign-column block on the received halo (beta = 1)."""
+
+    def __init__(self, A: CSR, fmt: str = "csr", group=None, **convert_opts):
+        if A.n_rows != A.n_cols:
+            raise ValueError("HaloSpMV needs a square matrix (x is owned like y)")
+        self.group = group
+        P = dist.get_world_size(group)
+        rank = dist.get_rank(group)
+        splits = partition(A, P)
+        self.layout = ShardLayout(splits, rank)
+        self.plan = HaloPlan(A.row_ptr, A.col, A.n_cols, splits, rank)
+        self.own = convert(spmv_slice_split(A, splits, rank, 0), fmt, **convert_opts)
+        self.foreign = convert(spmv_slice_split(A, splits, rank, 1, self.plan.colmap, self.plan.S), fmt,
+                               **convert_opts)
+        dev, self.dtype = A.row_ptr.device, A.val.dtype
+        self.x_own = torch.zeros(self.layout.rows, dtype=self.dtype, device=dev)
+        self.send = torch.zeros(self.plan.send_index.numel(), dtype=self.dtype, device=dev)
+        self.recv = torch.zeros(self.plan.recv_len, dtype=self.dtype, device=dev)
+
+    @property
+    def rows(self) -> int:
+        return self.layout.rows
+
+    def exchange_bytes(self) -> int:
+        return self.plan.exchange_bytes(self.recv.element_size())
+
+    def set_x(self, x_local: torch.Tensor):
+        self.x_own.copy_(x_local)
+        spmv_gather(self.x_own, self.plan.send_index, self.send)    # pack every receiver's halo
+
+    def run(self, alpha, beta, y_local: torch.Tensor, x_local: Optional[torch.Tensor] = None):
+        if x_local is not None:
+            self.set_x(x_local)
+        nccl = dist.get_backend(self.group) == "nccl"
+        work = self.plan.exchange(self.send, self.recv, self.group, async_op=nccl)
+        self.own.run(alpha, self.x_own, beta, y_local)              # overlaps the exchange
+        if work is not None:
+            work.wait()
+        self.foreign.run(alpha, self.recv, 1.0, y_local)
+        return y_local

@@ -184,3 +184,73 @@ def test_distspmv_nccl_world1_overlap(sp, compress):
         assert oracle.check_tolerance(yl.cpu().numpy(), ref, bound, 1e-12)[0]
     finally:
         dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("P", [2, 3, 5])
+@pytest.mark.parametrize("case", ["lap96", "rmat12"])
+@pytest.mark.parametrize("fmt", ["csr", "merge", "csr5", "ell"])
+def test_halo_virtual(sp, case, fmt, P):
+    """Halo exchange of P virtual ranks on one GPU: each rank's own
+    block (spmv_slice_split which=0) and foreign block remapped through its HaloPlan
+    colmap, halos packed by spmv_gather and moved by device copies standing in for the
+    all_to_all; integer regime, so bit-exact against the oracle."""
+    from paper_conf_ipps_nisassvs18_b200.dist import HaloPlan, ShardLayout
+    from paper_conf_ipps_nisassvs18_b200.spmv import spmv_gather, spmv_slice_split
+    A = matgen.rmat(12, seed=44, kind="int") if case == "rmat12" else matgen.laplacian5(96)
+    x = matgen.vector(A.n_cols, 44, 1, "int")
+    y = matgen.vector(A.n_rows, 44, 2, "int")
+    ref = oracle.spmv_csr(A, x, 2.0, -1.0, y)
+    dA = sp.CSR.from_host(A)
+    splits = sp.partition(dA, P)
+    lays = [ShardLayout(splits, k) for k in range(P)]
+    plans = [HaloPlan(dA.row_ptr, dA.col, A.n_cols, splits, k) for k in range(P)]
+    xd = torch.from_numpy(x).cuda()
+    sends = []
+    for k, lay in enumerate(lays):
+        buf = torch.empty(plans[k].send_index.numel(), dtype=torch.float64, device="cuda")
+        spmv_gather(lay.local_slice(xd).contiguous(), plans[k].send_index, buf)
+        sends.append(buf)
+    out = np.empty(A.n_rows)
+    for k, lay in enumerate(lays):
+        S = plans[k].S
+        recv = torch.zeros(P * S, dtype=torch.float64, device="cuda")
+        for o in range(P):                       # what all_to_all_single delivers
+            off = sum(plans[o].slots[:k])
+            recv[o * S: o * S + plans[o].slots[k]] = sends[o][off: off + plans[o].slots[k]]
+        try:
+            own = sp.convert(spmv_slice_split(dA, splits, k, 0), fmt)
+            foreign = sp.convert(spmv_slice_split(dA, splits, k, 1, plans[k].colmap, S), fmt)
+        except sp.SpmvError as e:
+            assert fmt == "ell" and e.status == 3
+            pytest.skip("ELL infeasible (A4)")
+        yl = torch.from_numpy(y[lay.r0:lay.r1].copy()).cuda()
+        own.run(2.0, lay.local_slice(xd).contiguous(), -1.0, yl)
+        foreign.run(2.0, recv, 1.0, yl)
+        out[lay.r0:lay.r1] = yl.cpu().numpy()
+    assert np.array_equal(out, ref)
+    if case == "lap96":
+        assert max(p.S for p in plans) <= 96        # one grid line per neighbour
+
+
+def test_halospmv_nccl_world1(sp):
+    import torch.distributed as dist
+    from paper_conf_ipps_nisassvs18_b200.dist import HaloSpMV
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK="0", WORLD_SIZE="1")
+    dist.init_process_group("nccl", device_id=torch.device("cuda", 0))
+    try:
+        A = matgen.laplacian5(80)
+        x = matgen.vector(A.n_cols, 45, 1)
+        y = matgen.vector(A.n_rows, 45, 2)
+        ref, bound = oracle.spmv_csr(A, x, 2.0, -1.0, y, with_bound=True)
+        H = HaloSpMV(sp.CSR.from_host(A), "csr")
+        yl = torch.from_numpy(y.copy()).cuda()
+        H.run(2.0, -1.0, yl, torch.from_numpy(x).cuda())
+        torch.cuda.synchronize()
+        ok, ratio, nbad = oracle.check_tolerance(yl.cpu().numpy(), ref, bound, 1e-12)
+        assert ok, (nbad, ratio)
+    finally:
+        dist.destroy_process_group()

@@ -29,8 +29,10 @@ def short(name):
     return n
 
 
-SPMV_KERNELS = ("k_coo", "k_ell", "k_csr_vector", "k_merge", "k_merge_persist", "k_csr5")
-B0_ARG = {"k_coo": 2, "k_ell": 1, "k_csr_vector": 3, "k_merge": 2, "k_merge_persist": 2, "k_csr5": 3}
+SPMV_KERNELS = ("k_coo", "k_ell", "k_csr_vector", "k_csr_rows", "k_merge", "k_merge_persist", "k_merge_rows",
+                "k_csr5")
+B0_ARG = {"k_coo": 2, "k_ell": 1, "k_csr_vector": 3, "k_csr_rows": 2, "k_merge": 2, "k_merge_persist": 2,
+          "k_merge_rows": 2, "k_csr5": 3}
 
 
 def targs(name):
@@ -127,12 +129,12 @@ def full(rep, out, traffic=None, formats=("coo", "ell", "csr", "hyb", "merge", "
         base = name.split("<")[0]
         seen[base] += 1
         ta = targs(name)
-        fmt = {"k_merge": "merge", "k_merge_persist": "merge", "k_csr5": "csr5"}.get(base)
+        fmt = {"k_merge": "merge", "k_merge_persist": "merge", "k_merge_rows": "merge", "k_csr5": "csr5"}.get(base)
         if base == "k_coo":
             fmt = "hyb" if ta[1] in ("1", "true") else "coo"
         elif base == "k_ell":
             fmt = "ell" if ("ell" in formats and seen[base] == 1) else "hyb"
-        elif base == "k_csr_vector" and seen[base] == 1 and "csr" in formats:
+        elif base in ("k_csr_vector", "k_csr_rows") and seen[base] == 1 and "csr" in formats:
             fmt = "csr"
         elif base == "k_csr_chunks" and "csr" in formats:
             fmt = "csr"
