@@ -1048,18 +1048,46 @@ struct MergeChunk {
     int c[8];
     V v[8];
 };
-template <typename V>
+// PAIRS: lane l holds chunk positions 2l + 64q and 2l + 64q + 1 (q < 4), so each load,
+// each product store and each x-gather instruction covers 64 consecutive positions
+// (conflict-free 512-byte stores; gathers of ~13 consecutive rows).  Else lane l holds
+// the 32-byte aligned run [8l, 8l + 8).
+template <typename V, bool PAIRS>
+__device__ __forceinline__ int chunk_pos(int lane, int e) {
+    return PAIRS ? 2 * lane + 64 * (e >> 1) + (e & 1) : 8 * lane + e;
+}
+template <typename V, bool PAIRS>
 __device__ __forceinline__ void merge_chunk_load(const int *__restrict__ col, const V *__restrict__ val, int64_t k0,
                                                  int64_t k1, MergeChunk<V> &ch, uint64_t pa) {
     const int lane = threadIdx.x & 31;
     const int off = (int)(k0 & 7);
-    if (lane * 8 - off < (int)(k1 - k0)) {
+    const int lim = (int)(k1 - k0) + off;                 // chunk positions < lim hold tile elements
+    if constexpr (PAIRS) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const int pos = 2 * lane + 64 * q;
+            if (pos < lim) {
+                const int2 c2 = ld_hint(reinterpret_cast<const int2 *>(col + (k0 - off) + pos), pa);
+                ch.c[2 * q] = c2.x;
+                ch.c[2 * q + 1] = c2.y;
+                if constexpr (sizeof(V) == 8) {
+                    const double2 v2 = ld_hint(reinterpret_cast<const double2 *>(val + (k0 - off) + pos), pa);
+                    ch.v[2 * q] = v2.x;
+                    ch.v[2 * q + 1] = v2.y;
+                } else {
+                    const float2 v2 = ld_hint(reinterpret_cast<const float2 *>(val + (k0 - off) + pos), pa);
+                    ch.v[2 * q] = v2.x;
+                    ch.v[2 * q + 1] = v2.y;
+                }
+            }
+        }
+    } else if (lane * 8 < lim) {
         ld256(col + (k0 - off) + lane * 8, ch.c, pa);
         VecLoad8<V>::load(val + (k0 - off) + lane * 8, ch.v, pa);
     }
 }
 
-template <typename V, typename IT, bool B0>
+template <typename V, typename IT, bool B0, bool PAIRS>
 __device__ __forceinline__ void
 merge_rows_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val, int64_t t,
                 int64_t r0, int64_t r1, int64_t k0, int64_t k1, const MergeChunk<V> &ch, const V *__restrict__ x,
@@ -1079,7 +1107,7 @@ merge_rows_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V 
     }
     // wait for the row ends before issuing the x gathers (measured: LAP4096 0.320 -> 0.298 ms)
     const bool ends_in = __all_sync(0xffffffffu, e_[0] >= 0 && e_[1] >= 0);   // every lane (no short circuit)
-    const bool any = any0 && ends_in;
+    (void)any0;
     double yv[2];
 #pragma unroll
     for (int q = 0; q < 2; ++q) {
@@ -1088,9 +1116,10 @@ merge_rows_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V 
     }
 #pragma unroll
     for (int e = 0; e < LI; e += 2) {
-        const double p0 = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)ch.v[e] * (double)ld_x(x + ch.c[e], px) : 0.0;
-        const double p1 = (any && (unsigned)(j0 + e + 1) < (unsigned)nnzt) ? (double)ch.v[e + 1] * (double)ld_x(x + ch.c[e + 1], px) : 0.0;
-        *reinterpret_cast<double2 *>(s_p + lane * LI + e) = make_double2(p0, p1);
+        const int pe = chunk_pos<V, PAIRS>(lane, e);      // chunk position of element e (pe + 1 of e + 1)
+        const double p0 = (ends_in && (unsigned)(pe - off) < (unsigned)nnzt) ? (double)ch.v[e] * (double)ld_x(x + ch.c[e], px) : 0.0;
+        const double p1 = (ends_in && (unsigned)(pe + 1 - off) < (unsigned)nnzt) ? (double)ch.v[e + 1] * (double)ld_x(x + ch.c[e + 1], px) : 0.0;
+        *reinterpret_cast<double2 *>(s_p + pe) = make_double2(p0, p1);
     }
     if (lane == 31) {                                     // positions past lane 31's chunk (< off row ends)
 #pragma unroll 1
@@ -1128,7 +1157,7 @@ merge_rows_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V 
 // takes tiles w, w + W, ... and the next tile's coordinates are loaded while the current
 // one runs; LIST = true: positions [i0, i1) of the tile order (SPMV_MERGE_SCHEDULE).
 // The identity schedule is measurably faster than the list (LAP4096: 0.298 vs 0.339 ms).
-template <typename V, typename IT, bool B0, int MB, bool LIST>
+template <typename V, typename IT, bool B0, int MB, bool LIST, bool PAIRS = true>
 __global__ void __launch_bounds__(kT, MB)
 k_merge_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
              const int64_t *__restrict__ crow, const int *__restrict__ order, int64_t i0, int64_t i1,
@@ -1140,8 +1169,8 @@ k_merge_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
     auto body = [&](int64_t t, int64_t r0, int64_t r1) {
         MergeChunk<V> ch;
         const int64_t k0 = merge_k(t, 256, r0, dmax), k1 = merge_k(t + 1, 256, r1, dmax);
-        merge_chunk_load(col, val, k0, k1, ch, pa);
-        merge_rows_tile<V, IT, B0>(rp, col, val, t, r0, r1, k0, k1, ch, x, y, alpha, beta, carry_row, carry_val,
+        merge_chunk_load<V, PAIRS>(col, val, k0, k1, ch, pa);
+        merge_rows_tile<V, IT, B0, PAIRS>(rp, col, val, t, r0, r1, k0, k1, ch, x, y, alpha, beta, carry_row, carry_val,
                                    s_p_all[wid], pa, px);
     };
     if constexpr (!LIST) {
@@ -1540,7 +1569,12 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
             const int *ord = (const int *)h->arr[SPMV_ARR_MERGE_TILE_ORDER].p;
             const int64_t nl = h->merge_lean, nt = h->merge_tiles;
             const unsigned gr = (unsigned)std::min<int64_t>(ceil_div<int64_t>(nl, kT / 32), (int64_t)h->ctx->sm_count * kMergeRowsMB);
-            if (nl == nt) {
+            static const bool pairs = [] { const char *e = getenv("SPMV_MERGE_PAIRS"); return !e || atoi(e) != 0; }();
+            if (nl == nt && !pairs) {
+                carveout(k_merge_rows<V, IT, B0, kMergeRowsMB, false, false>);
+                k_merge_rows<V, IT, B0, kMergeRowsMB, false, false><<<gr, kT, 0, s>>>(rp, col, val, cr, ord, 0, nt, dmax, x, y,
+                                                                               alpha, beta, crow, cval);
+            } else if (nl == nt) {
                 carveout(k_merge_rows<V, IT, B0, kMergeRowsMB, false>);
                 k_merge_rows<V, IT, B0, kMergeRowsMB, false><<<gr, kT, 0, s>>>(rp, col, val, cr, ord, 0, nt, dmax, x, y,
                                                                                alpha, beta, crow, cval);
