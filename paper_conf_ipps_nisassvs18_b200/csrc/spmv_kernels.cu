@@ -1469,8 +1469,9 @@ spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col
                               int64_t long_len = INT64_MAX) {
     if (n == 0) return SPMV_OK;
     // W <= 8: 32-row batches (A29) when col/val are 32-byte aligned (the chunk loads)
-    static const bool rows_on = [] { const char *e = getenv("SPMV_CSR_ROWS"); return !e || atoi(e) != 0; }();
-    if (w <= 8 && rows_on && ((((uintptr_t)col) | ((uintptr_t)val)) & 31) == 0) {
+    static const int rows_on = [] { const char *e = getenv("SPMV_CSR_ROWS"); return e ? atoi(e) : 1; }();
+    const int wmax = rows_on >= 8 ? rows_on : 8;          // experiment knob: SPMV_CSR_ROWS=16/32 widens it
+    if (w <= wmax && rows_on && ((((uintptr_t)col) | ((uintptr_t)val)) & 31) == 0) {
         const unsigned gr = (unsigned)std::min<int64_t>(ceil_div<int64_t>(n, kT), (int64_t)h->ctx->sm_count * kCsrRowsMB);
         if (long_len == INT64_MAX)
             k_csr_rows<V, IT, B0, kCsrRowsMB, false><<<gr, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len);

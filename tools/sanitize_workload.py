@@ -30,7 +30,13 @@ def main():
     n_launch = 0
     for kind, dt in (("f64", torch.float64), ("f32", torch.float32)):
         cases = edge_cases(kind)
-        for name in CASES:
+        # merge tile schedules (A28) and the CSR batch kernel's staged / unstaged batches (A29)
+        cases["lap64"] = matgen.laplacian5(64)
+        rng = np.random.default_rng(28)
+        lens = rng.integers(3, 8, 6000)
+        lens[[500, 4000]] = [900, 300]
+        cases["mixed_long"] = matgen.from_lengths(lens, 6000, seed=2801, kind=kind)
+        for name in CASES + ("lap64", "mixed_long"):
             A = cases[name]
             dA = sp.CSR.from_host(A, dtype=dt)
             sp.features(dA)
@@ -64,6 +70,14 @@ def main():
         S.spmv_gather(src, idx, dst)
         for which in (0, 1):
             S.spmv_slice_split(dA, splits, part, which)
+        # halo exchange plumbing: the foreign block through a HaloPlan colmap
+        from paper_conf_ipps_nisassvs18_b200.dist import HaloPlan
+        plan = HaloPlan(dA.row_ptr, dA.col, A.n_cols, splits, part)
+        fb = S.spmv_slice_split(dA, splits, part, 1, plan.colmap, plan.S)
+        hf = sp.convert(fb, "csr")
+        hf.run(1.0, torch.zeros(plan.recv_len, dtype=torch.float64, device="cuda"), 1.0,
+               torch.zeros(fb.n_rows, dtype=torch.float64, device="cuda"))
+        hf.destroy()
         del sl
     torch.cuda.synchronize()
     print(f"sanitize workload done: {n_launch} SpMV launches")
