@@ -458,6 +458,13 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
             v[s] = in ? ld_hint(val + e0 + s, pa) : (V)0;
         }
     }
+    // fp32: the x gathers before the y window loads (the products and the segmented sums
+    // need them first): LAP4096 0.321 -> 0.305 ms; fp64 measured 3 % slower that way
+    double p[8];
+    if constexpr (sizeof(V) == 4) {
+#pragma unroll
+        for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
+    }
     // rows around the tile (uniform loads)
     const int rf = __shfl_sync(0xffffffffu, r[0], 0);                       // tile's first row
     const int before = k0 > 0 ? __ldg(row + k0 - 1) : -1;                  // row before the tile
@@ -482,9 +489,10 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
 #pragma unroll
         for (int q = 0; q < kOutQ; ++q) s_acc[lane + 32 * q] = 0.0;
     }
-    double p[8];
+    if constexpr (sizeof(V) == 8) {
 #pragma unroll
-    for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
+        for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
+    }
     // rows past the window (sparse stretches: R-MAT's empty rows): the warp first writes
     // beta*y to all of them, 128 rows per step, coalesced; the tile's segments there then
     // add alpha*s (one more rounding of beta*y than the window path, within the bound)
