@@ -271,15 +271,15 @@ int ora_merge_class(int64_t n_rows, const int64_t *row_ptr, int64_t T,
 
 #define ORA_OMEGA 32
 
-/* A6: sigma = clamp(4*ceil(ceil(nnz_mu)/4), 4, 16). */
+/* A6 (B200 rule): sigma = 4 for ceil(nnz_mu) <= 3, 8 for 4, 12 above
+ * (multiples of 4 keep the lane runs 16-byte vectorizable; <= 16 fits the packing). */
 int64_t ora_csr5_sigma(int64_t n_rows, int64_t nnz)
 {
     if (n_rows <= 0) return 4;
     int64_t mu_ceil = (nnz + n_rows - 1) / n_rows;
-    int64_t s = 4 * ((mu_ceil + 3) / 4);
-    if (s < 4) s = 4;
-    if (s > 16) s = 16;
-    return s;
+    if (mu_ceil <= 3) return 4;
+    if (mu_ceil == 4) return 8;
+    return 12;
 }
 
 /* row_of[e] for every element: the row whose range contains e (a plain expansion). */

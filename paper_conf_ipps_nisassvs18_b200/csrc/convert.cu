@@ -490,9 +490,9 @@ spmv_status convert_t(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, const s
     }
     case SPMV_CSR5: {
         int64_t sigma = o->csr5_sigma;
-        if (sigma == 0) {   // A6
+        if (sigma == 0) {   // A6 (B200 rule): ceil(mu) <= 3 -> 4, == 4 -> 8, >= 5 -> 12
             int64_t mu = n > 0 ? ceil_div<int64_t>(nnz, n) : 1;
-            sigma = std::min<int64_t>(16, std::max<int64_t>(4, 4 * ceil_div<int64_t>(mu, 4)));
+            sigma = mu <= 3 ? 4 : (mu == 4 ? 8 : 12);
         }
         const int64_t W = 32 * sigma;
         const int64_t tiles = nnz / W;

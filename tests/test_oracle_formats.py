@@ -239,11 +239,14 @@ def test_slice_remap_reassembles_spmv(P):
 # ------------------------------------------------------------------ CSR5
 
 def test_csr5_sigma_rule():
-    """A6: sigma = clamp(4*ceil(ceil(nnz_mu)/4), 4, 16)."""
-    assert oracle.csr5_sigma(matgen.laplacian5(16)) == 8          # mu ~ 4.7 -> 5 -> 8
-    assert oracle.csr5_sigma(matgen.uniform_fixed(64, 64, 16)) == 16
+    """A6 (B200 rule, tools/csr5_sigma_sweep.py): sigma = 4 for ceil(nnz_mu) <= 3, 8 for
+    ceil(nnz_mu) = 4, 12 above."""
+    assert oracle.csr5_sigma(matgen.laplacian5(16)) == 12         # mu ~ 4.7 -> 5 -> 12
+    assert oracle.csr5_sigma(matgen.uniform_fixed(64, 64, 16)) == 12
     assert oracle.csr5_sigma(matgen.uniform_fixed(64, 64, 1)) == 4
-    assert oracle.csr5_sigma(matgen.uniform_fixed(64, 64, 40)) == 16
+    assert oracle.csr5_sigma(matgen.uniform_fixed(64, 64, 3)) == 4
+    assert oracle.csr5_sigma(matgen.uniform_fixed(64, 64, 4)) == 8
+    assert oracle.csr5_sigma(matgen.uniform_fixed(64, 64, 40)) == 12
 
 
 @pytest.mark.parametrize("i", range(N_CASES))
@@ -297,12 +300,15 @@ def test_csr5_decode_detects_corruption():
 def test_csr5_layout_is_lane_interleaved():
     """A6 layout: element e = t*W + l*sigma + s at t*W + (s//v)*32*v + l*v + s%v."""
     A = matgen.uniform_fixed(256, 4096, 16, seed=3)
-    e = oracle.csr5_encode(A, val_bytes=8)
-    sg, W = e["sigma"], 32 * e["sigma"]
-    for (t, l, s) in [(0, 0, 0), (0, 5, 3), (1, 31, 15), (2, 7, 9)]:
-        src = t * W + l * sg + s
-        assert e["col_perm"][t * W + (s // 4) * 128 + l * 4 + s % 4] == A.col[src]
-        assert e["val_perm"][t * W + (s // 2) * 64 + l * 2 + s % 2] == A.val[src]
+    for sigma, pts in ((16, [(0, 0, 0), (0, 5, 3), (1, 31, 15), (2, 7, 9)]),
+                       (12, [(0, 0, 0), (0, 5, 3), (1, 31, 11), (2, 7, 9)])):
+        e = oracle.csr5_encode(A, val_bytes=8, sigma=sigma)
+        sg, W = e["sigma"], 32 * e["sigma"]
+        assert sg == sigma
+        for (t, l, s) in pts:
+            src = t * W + l * sg + s
+            assert e["col_perm"][t * W + (s // 4) * 128 + l * 4 + s % 4] == A.col[src]
+            assert e["val_perm"][t * W + (s // 2) * 64 + l * 2 + s % 2] == A.val[src]
 
 
 # ------------------------------------------------------------------ features
