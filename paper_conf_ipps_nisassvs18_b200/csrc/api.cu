@@ -259,7 +259,7 @@ spmv_status spmv_info(const spmv_handle *h, spmv_handle_info *o) {
         // class from the tile order: both kept for export, not read by a run
         if (i != SPMV_ARR_MERGE_COORD_NZ && i != SPMV_ARR_MERGE_TILE_CLASS) fmt_bytes += h->arr[i].bytes;
     }
-    dev += h->carry_row.bytes + h->carry_val.bytes;
+    dev += h->carry_row.bytes + h->carry_val.bytes + h->sched.bytes;
     o->device_bytes = dev;
     // algorithmic bytes per run: the format's own arrays + x + y
     size_t V = h->dtype == SPMV_F64 ? 8 : 4;
@@ -308,6 +308,7 @@ spmv_status spmv_destroy(spmv_handle *h, void *stream) {
     dev_free(h->ctx, h->carry_row.p, h->carry_row.bytes, s);
     dev_free(h->ctx, h->carry_val.p, h->carry_val.bytes, s);
     dev_free(h->ctx, h->io_x.p, h->io_x.bytes, s);
+    dev_free(h->ctx, h->sched.p, h->sched.bytes, s);
     dev_free(h->ctx, h->io_y.p, h->io_y.bytes, s);
     delete h;
     return SPMV_OK;

@@ -557,6 +557,10 @@ spmv_status convert_t(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, const s
         break;
     }
     }
+    if (fmt == SPMV_CSR) {
+        h->sched.bytes = 16;
+        SPMV_TRY(dev_alloc(ctx, h->sched.bytes, s, &h->sched.p));
+    }
     if (h->n_carry > 0) {
         h->carry_row.bytes = h->n_carry * 8;
         h->carry_val.bytes = h->n_carry * 8;

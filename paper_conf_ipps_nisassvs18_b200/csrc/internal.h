@@ -80,6 +80,8 @@ struct spmv_handle {
     int64_t n_carry = 0;
     // spmv_run_host staging
     spmv::DevArray io_x, io_y;
+    // CSR-vector dynamic batch scheduler: one u64 counter, zeroed before every run
+    spmv::DevArray sched;
     int launches = 0;
 };
 

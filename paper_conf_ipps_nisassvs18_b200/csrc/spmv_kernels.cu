@@ -65,10 +65,11 @@ __global__ void k_scale(V *y, int64_t n, double beta) {
 // folded every kFold steps, A13) -- the paper's warp-per-row kernel for long rows.
 template <int W> struct VecCfg { static constexpr int U = W <= 8 ? 32 / (32 / W) : (W == 16 ? 4 : 2); };
 
-template <typename V, typename IT, int W, bool B0, int MB, bool CHUNKED>
+template <typename V, typename IT, int W, bool B0, int MB, bool CHUNKED, bool DYN = false>
 __global__ void __launch_bounds__(kT, MB)
 k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
-             const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta, int64_t long_len) {
+             const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta, int64_t long_len,
+             unsigned long long *__restrict__ sched = nullptr) {
     constexpr int G = 32 / W;
     constexpr int U = (VecCfg<W>::U * G > 32) ? 32 / G : VecCfg<W>::U;
     constexpr int R = G * U;                      // rows per warp iteration (<= 32)
@@ -78,15 +79,35 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
     const int64_t gwarp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
+    // DYN: warps take groups of kDynGroup batches from a global counter (zeroed before
+    // the launch), the next group requested one group ahead -- balances skewed rows (a
+    // static grid stride left R-MAT warps idle behind the slowest batch sequences)
+    constexpr int kDynGroup = 4;
+    unsigned long long ng = 0;
+    int j = 0;
     int64_t base = gwarp * R;
+    if constexpr (DYN) {
+        unsigned long long g0 = 0;
+        if (lane == 0) { g0 = atomicAdd(sched, 1ull); ng = atomicAdd(sched, 1ull); }
+        base = (int64_t)__shfl_sync(0xffffffffu, g0, 0) * (kDynGroup * R);
+    }
     IT nlo = 0, nhi = 0;                          // row pointers of the next batch (prefetched)
     if (base < n) {
         nlo = __ldg(rp + (base + lane < n ? base + lane : n));
         nhi = __ldg(rp + (base + R < n ? base + R : n));
     }
-    for (; base < n; base += nwarps * R) {
+    while (base < n) {
         const IT rp_lo = nlo, rp_hi = nhi;
-        const int64_t nb = base + nwarps * R;
+        int64_t nb = base + nwarps * R;
+        if constexpr (DYN) {
+            if (++j < kDynGroup) {
+                nb = base + R;
+            } else {
+                j = 0;
+                nb = (int64_t)__shfl_sync(0xffffffffu, ng, 0) * (kDynGroup * R);
+                if (lane == 0) ng = atomicAdd(sched, 1ull);
+            }
+        }
         if (nb < n) {                             // issue the next batch's row pointers now
             nlo = __ldg(rp + (nb + lane < n ? nb + lane : n));
             nhi = __ldg(rp + (nb + R < n ? nb + R : n));
@@ -195,6 +216,7 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
             if (!B0) o = fma(beta, yv, o);
             y[my_row] = (V)o;
         }
+        base = nb;
     }
 }
 
@@ -1493,8 +1515,21 @@ spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col
     const int g = grid_stride_blocks(h->ctx, threads, 16);
     // W <= 8: 4 CTAs/SM (64 registers; LAP4096 0.442 -> 0.384 ms); wider groups keep
     // 3 CTAs/SM (80 registers; R-MAT 24 at W = 16: 4 CTAs/SM 11 % slower)
+    // W >= 16 with the handle's scheduler counter: dynamic batch groups (skewed rows)
+    static const bool dyn_on = [] { const char *e = getenv("SPMV_CSR_DYN"); return !e || atoi(e) != 0; }();
+    // (only for row counts worth it: a resident grid -- 3 CTAs/SM -- with >= 4 groups per
+    // warp; small matrices keep the static stride, whose launch has no memset or atomics)
+    const int64_t resident_warps = (int64_t)h->ctx->sm_count * 3 * (kT / 32);
+    unsigned long long *sch = (dyn_on && h->sched.p && w >= 16 && n >= resident_warps * 4 * 4 * 32)
+                                  ? (unsigned long long *)h->sched.p : nullptr;
+    if (sch) SPMV_CUDA_TRY(cudaMemsetAsync(sch, 0, 8, s));
+    const int gd = sch ? (int)std::min<int64_t>(g, (int64_t)h->ctx->sm_count * 3) : g;
 #define SPMV_VEC(WW)                                                                                           \
-    if (long_len == INT64_MAX)                                                                            \
+    if (sch && long_len == INT64_MAX)                                                                     \
+        k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false, true><<<gd, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len, sch); \
+    else if (sch)                                                                                              \
+        k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true, true><<<gd, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len, sch); \
+    else if (long_len == INT64_MAX)                                                                            \
         k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false><<<g, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len); \
     else                                                                                                       \
         k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true><<<g, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len)

@@ -56,6 +56,17 @@ def main():
                         n_launch += h.launches()
                     h.destroy()
         torch.cuda.synchronize()
+    # CSR-vector with the dynamic batch scheduler (W >= 16, >= 1.8M rows): R-MAT scale 21
+    A = matgen.rmat(21, seed=21)
+    dA = sp.CSR.from_host(A)
+    h = sp.convert(dA, "csr")
+    xr = torch.from_numpy(matgen.vector(A.n_cols, 5, 1)).cuda()
+    yr = torch.from_numpy(matgen.vector(A.n_rows, 5, 2)).cuda()
+    h.run(1.0, xr, 1.0, yr)
+    n_launch += h.launches()
+    h.destroy()
+    del dA
+    torch.cuda.synchronize()
     # multi-GPU plumbing on one device: partition, remap, colmap, gather, own/foreign split
     A = matgen.rmat(12, seed=12)
     dA = sp.CSR.from_host(A)
