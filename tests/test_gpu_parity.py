@@ -620,3 +620,39 @@ def test_harness_record_cold_l2_and_scalar(sp):
             continue
         assert r["agree"] < 1e-12, f
         assert r["cold"]["cold_l2"] and r["cold"]["t_mean_ms"] > 0 and r["t_mean_ms"] > 0
+
+
+@pytest.mark.parametrize("name", ["lap64", "rmat12", "empty_runs", "big_skewed"])
+def test_cuda_graph_capture(sp, name):
+    """spmv_run is fully asynchronous and CUDA-graph capturable (include/spmv.h): every
+    format captured into a graph (beta = 0) replays bit-identically to the eager run --
+    including the CSR dynamic batch scheduler's counter reset (a >= 1.8M-row skewed
+    matrix) and the fix-up launches."""
+    A = matgen.rmat(21, seed=21) if name == "big_skewed" else case(name, "f64")
+    dA = to_dev(sp, A, torch.float64)
+    x = torch.from_numpy(matgen.vector(A.n_cols, 91, 1)).cuda()
+    fmts = ("csr", "merge", "csr5") if name == "big_skewed" else ("coo", "ell", "csr", "hyb", "merge", "csr5")
+    for fmt in fmts:
+        try:
+            h = sp.convert(dA, fmt)
+        except sp.SpmvError as e:
+            assert e.status == 3
+            continue
+        y_eager = torch.full((A.n_rows,), float("nan"), dtype=torch.float64, device="cuda")
+        h.run(1.25, x, 0.0, y_eager)
+        y_graph = torch.full((A.n_rows,), float("nan"), dtype=torch.float64, device="cuda")
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s):
+            h.run(1.25, x, 0.0, y_graph)                       # warm-up on the capture stream
+        torch.cuda.current_stream().wait_stream(s)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            h.run(1.25, x, 0.0, y_graph)
+        y_graph.fill_(float("nan"))
+        for _ in range(2):
+            g.replay()
+        torch.cuda.synchronize()
+        assert torch.equal(y_graph, y_eager), fmt
+        del g
+        h.destroy()
