@@ -30,6 +30,7 @@ constexpr int kIPT = kItemsPerThread;
 constexpr int kWIPT = kWarpItemsPerLane;
 constexpr int kMinBlocks = 4;   // 4 CTAs x 256 threads per SM: <= 64 registers
 constexpr int kFold = 256;
+constexpr int kSubMax = 256;  // CSR-vector: longest remainder walked by a lane subgroup (else whole warp)
 constexpr int kMergeRowsMB = 4;   // k_merge_rows CTAs per SM
 constexpr int kCsrRowsMB = 4;     // k_csr_rows CTAs per SM   // sequential steps per accumulator before folding (A13)
 
@@ -45,6 +46,15 @@ template <typename V, bool B0>
 __device__ __forceinline__ void y_beta(V *y, int64_t r, double beta) {
     y[r] = B0 ? (V)0 : (V)(beta * (double)y[r]);
 }
+
+// ------------------------------------------------------------------ PDL (CSR long rows)
+// The CSR row kernel is launched programmatically dependent on k_csr_chunks (A25), which
+// triggers its dependents at entry: the row kernel's CTAs fill the SMs beside the chunk
+// CTAs (the two are independent), and each row-kernel thread waits for the chunk grid
+// before exiting, so the fix-up launched after it sees the chunk carries.  Both are
+// no-ops when the kernel is launched without the attribute.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
 // ------------------------------------------------------------------ alpha == 0
 
@@ -180,7 +190,45 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
             const IT my_b = __shfl_sync(0xffffffffu, rp_lo, (lane + 1) & 31);
             const IT my_e = lane + 1 < R ? my_b : rp_hi;
             const int64_t my_len = (int64_t)my_e - (int64_t)my_a;
-            unsigned more = __ballot_sync(0xffffffffu, lane < R && base + lane < n && my_len > W && (!CHUNKED || my_len <= long_len));
+            const bool is_long = lane < R && base + lane < n && my_len > W && (!CHUNKED || my_len <= long_len);
+            // remainders of at most kSubMax: all such rows of the batch at once, a subgroup
+            // of SW = 32 / next_pow2(count) lanes per row, 8 predicated loads per lane per
+            // step -- one gather round trip for the batch instead of one per row (R-MAT's
+            // many rows a little longer than W)
+            const unsigned few = __ballot_sync(0xffffffffu, is_long && my_len - W <= kSubMax);
+            unsigned more = __ballot_sync(0xffffffffu, is_long) & ~few;
+            if (few) {
+                const int nl = __popc(few);
+                const int lg = nl > 1 ? 32 - __clz(nl - 1) : 0;
+                const int SW = 32 >> lg;
+                const int sg = lane >> (5 - lg), sl = lane & (SW - 1);
+                const int ri = sg < nl ? (int)__fns(few, 0, sg + 1) : 0;
+                const int64_t ra = (int64_t)__shfl_sync(0xffffffffu, my_a, ri) + W;
+                const int64_t re = (int64_t)__shfl_sync(0xffffffffu, my_e, ri);
+                const int64_t rb = sg < nl ? re : ra;
+                double acc[8];
+#pragma unroll
+                for (int q = 0; q < 8; ++q) acc[q] = 0.0;
+                for (int64_t k = ra + sl; k < rb; k += 8 * SW) {
+                    int d[8];
+                    V w[8];
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) {
+                        const bool in = k + q * SW < rb;
+                        d[q] = in ? ld_hint(col + k + q * SW, pa) : -1;
+                        w[q] = in ? ld_hint(val + k + q * SW, pa) : (V)0;
+                    }
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) if (d[q] >= 0) acc[q] += (double)w[q] * (double)ld_x(x + d[q], px);
+                }
+                double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
+                for (int o = SW >> 1; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+                const int wi = g * U + (sub < U ? sub : 0);           // this lane's row (writer lanes)
+                const bool wmine = sub < U && ((few >> wi) & 1u);
+                const int src = (__popc(few & ((1u << wi) - 1u)) << (5 - lg)) & 31;
+                const double got = __shfl_sync(0xffffffffu, part, src);
+                if (wmine) mine += got;
+            }
             while (more) {
                 const int i = __ffs(more) - 1;
                 more &= more - 1;
@@ -218,6 +266,7 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
         }
         base = nb;
     }
+    pdl_wait();   // PDL after k_csr_chunks: exit only once the chunk grid is done (else a no-op)
 }
 
 // ------------------------------------------------------------------ CSR long-row chunks (A25)
@@ -229,6 +278,7 @@ __global__ void __launch_bounds__(kT)
 k_csr_chunks(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
              const int64_t *__restrict__ crow, const int64_t *__restrict__ clo, int64_t nch, int64_t C,
              const V *__restrict__ x, int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
+    pdl_trigger();
     const int lane = threadIdx.x & 31;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
     for (int64_t c = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; c < nch;
@@ -772,6 +822,7 @@ k_csr_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
             y[b + lane] = (V)o;
         }
     }
+    pdl_wait();   // PDL after k_csr_chunks: exit only once the chunk grid is done (else a no-op)
 }
 
 // ------------------------------------------------------------------ merge-based CSR (K7/G11)
@@ -1493,10 +1544,38 @@ spmv_status launch_ell(spmv_handle *h, const V *x, V *y, double alpha, double be
     return SPMV_OK;
 }
 
+// kT-thread launch of `k` on `s`; pdl = programmatic dependent launch on the kernel
+// before it in the stream (cudaLaunchAttributeProgrammaticStreamSerialization)
+template <typename... KArgs, typename... Args>
+cudaError_t launch_k(void (*k)(KArgs...), unsigned grid, cudaStream_t s, bool pdl, Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(kT);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = pdl ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
+}
+
+// the CSR-vector dynamic batch counter for this run, or nullptr: W >= 16 with the
+// handle's scheduler counter, and only for row counts worth it (a resident grid --
+// 3 CTAs/SM -- with >= 4 groups per warp; small matrices keep the static stride, whose
+// launch has no memset or atomics)
+inline unsigned long long *csr_sched(const spmv_handle *h, int64_t n, int w) {
+    static const bool dyn_on = [] { const char *e = getenv("SPMV_CSR_DYN"); return !e || atoi(e) != 0; }();
+    const int64_t resident_warps = (int64_t)h->ctx->sm_count * 3 * (kT / 32);
+    return (dyn_on && h->sched.p && w >= 16 && n >= resident_warps * 4 * 4 * 32) ? (unsigned long long *)h->sched.p
+                                                                                 : nullptr;
+}
+
 template <typename V, typename IT, bool B0>
 spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col, const V *val, const V *x, V *y,
                               int64_t n, int w, double alpha, double beta, cudaStream_t s,
-                              int64_t long_len = INT64_MAX) {
+                              int64_t long_len = INT64_MAX, bool pdl = false) {
     if (n == 0) return SPMV_OK;
     // W <= 8: 32-row batches (A29) when col/val are 32-byte aligned (the chunk loads)
     static const int rows_on = [] { const char *e = getenv("SPMV_CSR_ROWS"); return e ? atoi(e) : 1; }();
@@ -1504,10 +1583,9 @@ spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col
     if (w <= wmax && rows_on && ((((uintptr_t)col) | ((uintptr_t)val)) & 31) == 0) {
         const unsigned gr = (unsigned)std::min<int64_t>(ceil_div<int64_t>(n, kT), (int64_t)h->ctx->sm_count * kCsrRowsMB);
         if (long_len == INT64_MAX)
-            k_csr_rows<V, IT, B0, kCsrRowsMB, false><<<gr, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len);
+            SPMV_CUDA_TRY(launch_k(k_csr_rows<V, IT, B0, kCsrRowsMB, false>, gr, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len));
         else
-            k_csr_rows<V, IT, B0, kCsrRowsMB, true><<<gr, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len);
-        SPMV_LAUNCH_CHECK();
+            SPMV_CUDA_TRY(launch_k(k_csr_rows<V, IT, B0, kCsrRowsMB, true>, gr, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len));
         return SPMV_OK;
     }
     // 16 CTAs (4096 threads) per SM of grid-stride warps
@@ -1515,24 +1593,19 @@ spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col
     const int g = grid_stride_blocks(h->ctx, threads, 16);
     // W <= 8: 4 CTAs/SM (64 registers; LAP4096 0.442 -> 0.384 ms); wider groups keep
     // 3 CTAs/SM (80 registers; R-MAT 24 at W = 16: 4 CTAs/SM 11 % slower)
-    // W >= 16 with the handle's scheduler counter: dynamic batch groups (skewed rows)
-    static const bool dyn_on = [] { const char *e = getenv("SPMV_CSR_DYN"); return !e || atoi(e) != 0; }();
-    // (only for row counts worth it: a resident grid -- 3 CTAs/SM -- with >= 4 groups per
-    // warp; small matrices keep the static stride, whose launch has no memset or atomics)
-    const int64_t resident_warps = (int64_t)h->ctx->sm_count * 3 * (kT / 32);
-    unsigned long long *sch = (dyn_on && h->sched.p && w >= 16 && n >= resident_warps * 4 * 4 * 32)
-                                  ? (unsigned long long *)h->sched.p : nullptr;
-    if (sch) SPMV_CUDA_TRY(cudaMemsetAsync(sch, 0, 8, s));
+    unsigned long long *sch = csr_sched(h, n, w);
+    if (sch && !pdl) SPMV_CUDA_TRY(cudaMemsetAsync(sch, 0, 8, s));   // pdl: zeroed before the chunk launch
     const int gd = sch ? (int)std::min<int64_t>(g, (int64_t)h->ctx->sm_count * 3) : g;
 #define SPMV_VEC(WW)                                                                                           \
-    if (sch && long_len == INT64_MAX)                                                                     \
-        k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false, true><<<gd, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len, sch); \
+    if (sch && long_len == INT64_MAX)                                                                          \
+        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false, true>, gd, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len, sch)); \
     else if (sch)                                                                                              \
-        k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true, true><<<gd, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len, sch); \
+        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true, true>, gd, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len, sch)); \
     else if (long_len == INT64_MAX)                                                                            \
-        k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false><<<g, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len); \
+        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false>, g, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len, nosch)); \
     else                                                                                                       \
-        k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true><<<g, kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta, long_len)
+        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true>, g, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len, nosch))
+    unsigned long long *nosch = nullptr;
     switch (w) {
     case 1: case 2: SPMV_VEC(2); break;
     case 4: SPMV_VEC(4); break;
@@ -1558,14 +1631,27 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
     case SPMV_CSR:
     {
         if (h->csr_chunks == 0) return launch_csr_vector<V, IT, B0>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s);
-        SPMV_TRY((launch_csr_vector<V, IT, B0>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s,
-                                               2 * h->csr_chunk)));
+        // long-row chunks first, the row kernel programmatically dependent on them (PDL):
+        // the two are independent and run side by side; the chunk grid is one resident
+        // wave of chunk_ctas (2) CTAs/SM so that the row kernel's CTAs start at once beside it
+        static const bool pdl_on = [] { const char *e = getenv("SPMV_CSR_PDL"); return !e || atoi(e) != 0; }();
+        static const int chunk_ctas = [] { const char *e = getenv("SPMV_CSR_CHUNK_CTAS"); return e ? std::max(1, atoi(e)) : 2; }();
+        if (pdl_on) {
+            if (unsigned long long *sch = csr_sched(h, n, (int)h->vec_w)) SPMV_CUDA_TRY(cudaMemsetAsync(sch, 0, 8, s));
+        } else {
+            SPMV_TRY((launch_csr_vector<V, IT, B0>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s,
+                                                   2 * h->csr_chunk)));
+        }
         const int64_t warps = h->csr_chunks;
-        const unsigned gc = (unsigned)std::min<int64_t>(ceil_div<int64_t>(warps, kT / 32), (int64_t)h->ctx->sm_count * 16);
+        const unsigned gc = (unsigned)std::min<int64_t>(ceil_div<int64_t>(warps, kT / 32),
+                                                        (int64_t)h->ctx->sm_count * (pdl_on ? chunk_ctas : 16));
         k_csr_chunks<V, IT><<<gc, kT, 0, s>>>(rp, col, val, (const int64_t *)h->arr[SPMV_ARR_CSR_CHUNK_ROW].p,
                                               (const int64_t *)h->arr[SPMV_ARR_CSR_CHUNK_LO].p, h->csr_chunks,
                                               h->csr_chunk, x, crow, cval);
         SPMV_LAUNCH_CHECK();
+        if (pdl_on)
+            SPMV_TRY((launch_csr_vector<V, IT, B0>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s,
+                                                   2 * h->csr_chunk, true)));
         return launch_fixup<V>(h, y, alpha, s);
     }
     case SPMV_CSR_SCALAR:
