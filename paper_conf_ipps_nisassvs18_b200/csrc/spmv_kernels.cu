@@ -266,7 +266,10 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
         }
         base = nb;
     }
-    pdl_wait();   // PDL after k_csr_chunks: exit only once the chunk grid is done (else a no-op)
+    // PDL after k_csr_chunks (chunked handles only): exit only once the chunk grid is
+    // done.  Not compiled into the unchunked kernels: even with nothing to wait for it
+    // cost LAP4096 7-15 %
+    if constexpr (CHUNKED) pdl_wait();
 }
 
 // ------------------------------------------------------------------ CSR long-row chunks (A25)
@@ -822,7 +825,10 @@ k_csr_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
             y[b + lane] = (V)o;
         }
     }
-    pdl_wait();   // PDL after k_csr_chunks: exit only once the chunk grid is done (else a no-op)
+    // PDL after k_csr_chunks (chunked handles only): exit only once the chunk grid is
+    // done.  Not compiled into the unchunked kernels: even with nothing to wait for it
+    // cost LAP4096 7-15 %
+    if constexpr (CHUNKED) pdl_wait();
 }
 
 // ------------------------------------------------------------------ merge-based CSR (K7/G11)

@@ -656,3 +656,45 @@ def test_cuda_graph_capture(sp, name):
         assert torch.equal(y_graph, y_eager), fmt
         del g
         h.destroy()
+
+
+_PDL_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import matgen
+import paper_conf_ipps_nisassvs18_b200 as sp
+outs = []
+for A in (matgen.rmat(21, seed=21), matgen.from_lengths(np.r_[np.ones(3000, np.int64), [40000], np.ones(3000, np.int64)], 50000, seed=3)):
+    dA = sp.CSR.from_host(A, dtype=torch.float64)
+    h = sp.convert(dA, "csr")
+    x = torch.from_numpy(matgen.vector(A.n_cols, 17, 1)).cuda()
+    y = torch.from_numpy(matgen.vector(A.n_rows, 17, 2)).cuda()
+    h.run(1.5, x, -0.5, y)
+    torch.cuda.synchronize()
+    outs.append(y.cpu().numpy())
+    h.destroy()
+np.save(sys.argv[2], np.concatenate(outs))
+"""
+
+
+def test_csr_pdl_matches_serial(sp, tmp_path):
+    """A25's launch order -- long-row chunk kernel first, the row kernel a programmatic
+    dependent launch beside it -- changes no arithmetic: y is bit-identical to the serial
+    order (SPMV_CSR_PDL=0, row kernel then chunks), on R-MAT 21 (dynamic batch scheduler
+    + chunks) and a short-row matrix with one 40,000-nonzero row; both within the bound."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    res = {}
+    for pdl in ("1", "0"):
+        out = tmp_path / f"y_pdl{pdl}.npy"
+        env = dict(os.environ, SPMV_CSR_PDL=pdl)
+        subprocess.run([sys.executable, "-c", _PDL_SCRIPT, root, str(out)], env=env, check=True, timeout=600)
+        res[pdl] = np.load(out)
+    assert np.array_equal(res["1"].view(np.uint64), res["0"].view(np.uint64))
+    A = matgen.rmat(21, seed=21)
+    x, y0 = matgen.vector(A.n_cols, 17, 1), matgen.vector(A.n_rows, 17, 2)
+    ref, bound = oracle.spmv_csr(A, x, 1.5, -0.5, y0, with_bound=True)
+    ok, ratio, nbad = oracle.check_tolerance(res["1"][:A.n_rows], ref, bound, TOL[torch.float64])
+    assert ok, f"R-MAT 21 CSR (PDL): {nbad} bad rows, max ratio {ratio}"
