@@ -92,7 +92,9 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
     // DYN: warps take groups of kDynGroup batches from a global counter (zeroed before
     // the launch), the next group requested one group ahead -- balances skewed rows (a
     // static grid stride left R-MAT warps idle behind the slowest batch sequences)
-    constexpr int kDynGroup = 4;
+    // (batches per group: fp64 2, fp32 4 -- R-MAT 24 fp64 group 4 1.82 ms, 2 1.79, 8 1.84;
+    // fp32 group 4 1.60, 2 1.70; R-MAT 22 fp64 0.50 / 0.47 / 0.56)
+    constexpr int kDynGroup = sizeof(V) == 8 ? 2 : 4;
     unsigned long long ng = 0;
     int j = 0;
     int64_t base = gwarp * R;
