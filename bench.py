@@ -274,13 +274,18 @@ def run_ours(args):
 
     formats = [f for f in args.formats.split(",") if f] if args.formats else list(sp.PAPER_FORMATS)
 
-    # ---- features (a2), timed once
-    fe0, fe1 = ev(), ev()
-    fe0.record(stream)
+    # ---- features (a2): one untimed call (ctx state, module load), then the warm median of
+    # `feat_reps` blocking calls (one kernel + one 112-byte readback each)
     feats = sp.features(dA)
-    fe1.record(stream)
     torch.cuda.synchronize()
-    feat_ms = fe0.elapsed_time(fe1)
+    feat_t = []
+    for _ in range(args.feat_reps):
+        t0 = time.perf_counter()
+        sp.features(dA)
+        feat_t.append(time.perf_counter() - t0)
+    feat_t.sort()
+    feat_ms = feat_t[len(feat_t) // 2] * 1e3
+    feat_bytes = (A.n_rows + 1) * dA.row_ptr.element_size() + 4 * A.nnz
 
     # ---- partition (a14) for N > 1: this rank's rows, columns remapped to gathered-x slots
     # (DistSpMV: merge-path row splits, shard, optional compressed exchange)
@@ -306,7 +311,7 @@ def run_ours(args):
         c0, c1 = ev(), ev()
         c0.record(stream)
         try:
-            handles[f] = sp.convert(local_A, f)
+            handles[f] = sp.convert(local_A, f, features=feats if local_A is dA else None)
         except sp.SpmvError as e:
             if e.status in (3, 4):
                 na[f] = e.name
@@ -519,7 +524,11 @@ def run_ours(args):
                                                    else dsp.exchange_bytes() if dsp is not None else 0)},
             "per_format": per_format, "best_format": best,
             "roofline": roof(dom), "roofline_best": roof(best),
-            "features": {"ms": feat_ms, "gbs": (4 * A.nnz + 8 * (A.n_rows + 1)) / (feat_ms * 1e-3) / 1e9,
+            "features": {"ms": feat_ms, "ms_min": feat_t[0] * 1e3, "bytes": feat_bytes,
+                         "gbs": feat_bytes / (feat_ms * 1e-3) / 1e9,
+                         "frac_of_peak": feat_bytes / (feat_ms * 1e-3) / 1e9 / peak,
+                         "timing": f"warm median of {len(feat_t)} blocking spmv_features calls (wall clock: "
+                                   "one kernel launch + one 112-byte readback each)",
                          "values": {k: feats[k] for k in sp.PAPER_FEATURES}},
             "label6": best, "gpu_launches": launches_per_step * args.steps,
             "clocks": clk.summary(), "e2e": e2e, "cpu_baseline": cpu,
@@ -559,6 +568,7 @@ def main():
     ap.add_argument("--overlap", action="store_true",
                     help="N > 1: own-column blocks run while the x all-gather is in flight")
     ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--feat-reps", type=int, default=20, help="warm spmv_features calls timed")
     ap.add_argument("--e2e-serial", action="store_true", help="e2e: run the formats' host calls in turn")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0)

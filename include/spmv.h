@@ -35,7 +35,7 @@ extern "C" {
 #pragma GCC visibility push(default)
 #endif
 
-#define SPMV_ABI_VERSION 2
+#define SPMV_ABI_VERSION 3
 
 typedef enum {
     SPMV_OK = 0,
@@ -119,9 +119,11 @@ typedef struct {
     uint64_t sum_len2, sum_nnzb2, sum_snzb2;              /* exact sums behind the sigmas */
 } spmv_features_t;
 
-/* One O(nnz) device pass over row_ptr + col_idx (vals are not read), then one
- * device->host readback: BLOCKS on `stream`.  Returns SPMV_ERR_NOT_CANONICAL
- * for a non-canonical matrix (out_host is then unspecified). */
+/* One kernel launch reads row_ptr and col_idx once each (vals are not read; DESIGN.md
+ * §4 "Features"), then one 112-byte device->host readback: BLOCKS on `stream`.  No
+ * allocation after the ctx's first call (device state is ctx-owned and reset by the
+ * kernel; concurrent callers on one ctx are serialised).  Returns
+ * SPMV_ERR_NOT_CANONICAL for a non-canonical matrix (out_host is then unspecified). */
 spmv_status spmv_features(spmv_ctx *ctx, const spmv_csr *A, void *stream,
                           spmv_features_t *out_host);
 
@@ -131,7 +133,8 @@ typedef struct {
     int hyb_rule;          /* 0 = ceil(nnz/n_rows) (default; "nnz_mu, which we
                               use", A2), 1 = floor, 2 = the max(4096, rows/3)-style rule   */
     int64_t hyb_width;     /* >= 0 overrides hyb_rule; < 0 = use the rule                 */
-    int csr5_sigma;        /* 0 = A6 rule clamp(4*ceil(ceil(nnz_mu)/4), 4, 16); else 4..16, %4 */
+    int csr5_sigma;        /* 0 = A6 rule (B200 revision): 4 if ceil(nnz_mu) <= 3, 8 if it is 4,
+                              12 above; else 4, 8, 12 or 16                                 */
     int merge_items;       /* merge-path items per CTA (0 = default); recorded in info     */
     int vector_width;      /* CSR-vector lanes per row (0 = A5 rule), power of two 1..32  */
     size_t max_bytes;      /* ELL/HYB guard (0 = min(1/2 free memory, max(8x the CSR bytes,
@@ -144,6 +147,13 @@ typedef struct {
     int64_t csr_chunk;     /* CSR long-row split (A25): rows longer than 2*csr_chunk are cut
                               into csr_chunk-nonzero chunks, each reduced by its own warp and
                               added by the fix-up; 0 = default 512, < 0 = never split     */
+    const spmv_features_t *features;
+                           /* optional HOST pointer: the spmv_features() result of THIS matrix
+                              (same arrays, unchanged since).  The conversion then reuses it
+                              (nnz_max, hyb_width_cusp) and skips its own feature/validation
+                              pass; dimensions must match A (else SPMV_ERR_INVALID_ARG).
+                              Features of another matrix are undefined behaviour.  NULL =
+                              validate here (one feature pass, one readback).              */
 } spmv_convert_opts;
 
 /* Fill `opts` with the defaults (all rules as above). */

@@ -51,6 +51,27 @@ void dev_free(spmv_ctx *ctx, void *p, size_t bytes, cudaStream_t s) {
     else cudaFreeAsync(p, s);
 }
 
+// Every entry point that touches the device runs on the ctx's device and leaves the
+// caller's current device as it found it.
+struct DeviceGuard {
+    int prev = -1;
+    cudaError_t err = cudaSuccess;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) { cudaGetLastError(); prev = -1; }
+        if (prev != dev) err = cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+};
+#define SPMV_ON_DEVICE(dev)                                                        \
+    DeviceGuard _dg(dev);                                                          \
+    if (_dg.err != cudaSuccess) {                                                  \
+        set_error(std::string("cudaSetDevice: ") + cudaGetErrorString(_dg.err));   \
+        return SPMV_ERR_CUDA;                                                      \
+    }
+
 static spmv_status check_csr(const spmv_csr *A) {
     if (!A) { set_error("A is NULL"); return SPMV_ERR_INVALID_ARG; }
     if (A->n_rows < 0 || A->n_cols < 0 || A->nnz < 0) { set_error("negative dimension"); return SPMV_ERR_INVALID_ARG; }
@@ -107,7 +128,7 @@ spmv_status spmv_init(int device, const spmv_allocator *alloc, spmv_ctx **out) {
                   std::to_string(prop.minor));
         return SPMV_ERR_UNSUPPORTED;
     }
-    SPMV_CUDA_TRY(cudaSetDevice(device));
+    SPMV_ON_DEVICE(device);
     spmv_ctx *c = new (std::nothrow) spmv_ctx();
     if (!c) return SPMV_ERR_NO_MEMORY;
     c->device = device;
@@ -122,6 +143,11 @@ spmv_status spmv_init(int device, const spmv_allocator *alloc, spmv_ctx **out) {
 }
 
 spmv_status spmv_finalize(spmv_ctx *ctx) {
+    if (!ctx) return SPMV_OK;
+    {
+        DeviceGuard dg(ctx->device);
+        feature_state_free(ctx);
+    }
     delete ctx;
     return SPMV_OK;
 }
@@ -137,7 +163,7 @@ spmv_status spmv_features(spmv_ctx *ctx, const spmv_csr *A, void *stream, spmv_f
     NvtxRange nv("spmv_features");
     if (!ctx || !out) { set_error("NULL ctx/out"); return SPMV_ERR_INVALID_ARG; }
     SPMV_TRY(check_csr(A));
-    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    SPMV_ON_DEVICE(ctx->device);
     FeatureSums fs;
     int64_t cusp = 0;
     SPMV_TRY(feature_pass(ctx, A, as_stream(stream), 1, &fs, &cusp));
@@ -174,7 +200,7 @@ spmv_status spmv_convert(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A,
         set_error("vector_width must be a power of two <= 32");
         return SPMV_ERR_INVALID_ARG;
     }
-    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    SPMV_ON_DEVICE(ctx->device);
     spmv_handle *h = new (std::nothrow) spmv_handle();
     if (!h) return SPMV_ERR_NO_MEMORY;
     h->ctx = ctx;
@@ -206,6 +232,7 @@ spmv_status spmv_run(spmv_handle *h, const void *alpha, const void *x, const voi
     double a, b;
     if (h->dtype == SPMV_F64) { a = *(const double *)alpha; b = *(const double *)beta; }
     else { a = *(const float *)alpha; b = *(const float *)beta; }
+    SPMV_ON_DEVICE(h->ctx->device);
     NvtxRange nv(kRunNames[h->fmt]);
     return run_impl(h, a, b, x, y, as_stream(stream));
 }
@@ -215,6 +242,7 @@ spmv_status spmv_run_host(spmv_handle *h, const void *alpha, const void *x_host,
     if (!h || !alpha || !beta) { set_error("NULL handle/alpha/beta"); return SPMV_ERR_INVALID_ARG; }
     size_t V = h->dtype == SPMV_F64 ? 8 : 4;
     cudaStream_t s = as_stream(stream);
+    SPMV_ON_DEVICE(h->ctx->device);
     size_t bx = (size_t)h->n_cols * V, by = (size_t)h->n_rows * V;
     if (!h->io_x.p && bx) { SPMV_TRY(dev_alloc(h->ctx, bx, s, &h->io_x.p)); h->io_x.bytes = bx; }
     if (!h->io_y.p && by) { SPMV_TRY(dev_alloc(h->ctx, by, s, &h->io_y.p)); h->io_y.bytes = by; }
@@ -295,6 +323,7 @@ spmv_status spmv_export(const spmv_handle *h, spmv_array_id id, void *dst, size_
     }
     if (cap < a.bytes || !dst) { set_error("destination too small"); return SPMV_ERR_INVALID_ARG; }
     cudaStream_t s = as_stream(stream);
+    SPMV_ON_DEVICE(h->ctx->device);
     SPMV_CUDA_TRY(cudaMemcpyAsync(dst, a.p, a.bytes, cudaMemcpyDeviceToHost, s));
     SPMV_CUDA_TRY(cudaStreamSynchronize(s));
     return SPMV_OK;
@@ -303,6 +332,7 @@ spmv_status spmv_export(const spmv_handle *h, spmv_array_id id, void *dst, size_
 spmv_status spmv_destroy(spmv_handle *h, void *stream) {
     if (!h) return SPMV_OK;
     cudaStream_t s = as_stream(stream);
+    DeviceGuard dg(h->ctx->device);
     for (int i = 0; i < kMaxArrays; ++i)
         if (h->arr[i].owned && h->arr[i].p) dev_free(h->ctx, h->arr[i].p, h->arr[i].bytes + 64, s);
     dev_free(h->ctx, h->carry_row.p, h->carry_row.bytes, s);
@@ -318,7 +348,7 @@ spmv_status spmv_partition(spmv_ctx *ctx, const spmv_csr *A, int nparts, void *s
     NvtxRange nv("spmv_partition");
     if (!ctx || !splits || nparts <= 0) { set_error("bad ctx/splits/nparts"); return SPMV_ERR_INVALID_ARG; }
     SPMV_TRY(check_csr(A));
-    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    SPMV_ON_DEVICE(ctx->device);
     return partition_impl(ctx, A, nparts, as_stream(stream), splits);
 }
 
@@ -326,7 +356,7 @@ spmv_status spmv_slice_size(spmv_ctx *ctx, const spmv_csr *A, const int64_t *spl
                             void *stream, int64_t *rows, int64_t *nnz, int64_t *slot) {
     if (!ctx || !splits || nparts <= 0 || part < 0 || part >= nparts) { set_error("bad args"); return SPMV_ERR_INVALID_ARG; }
     SPMV_TRY(check_csr(A));
-    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    SPMV_ON_DEVICE(ctx->device);
     return slice_size_impl(ctx, A, splits, nparts, part, as_stream(stream), rows, nnz, slot);
 }
 
@@ -335,7 +365,7 @@ spmv_status spmv_slice_remap(spmv_ctx *ctx, const spmv_csr *A, const int64_t *sp
     if (!ctx || !splits || nparts <= 0 || part < 0 || part >= nparts || !rp_out) { set_error("bad args"); return SPMV_ERR_INVALID_ARG; }
     SPMV_TRY(check_csr(A));
     if (A->n_rows != A->n_cols) { set_error("slice_remap needs a square matrix"); return SPMV_ERR_INVALID_ARG; }
-    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    SPMV_ON_DEVICE(ctx->device);
     return slice_remap_impl(ctx, A, splits, nparts, part, as_stream(stream), rp_out, col_out, val_out);
 }
 
@@ -344,7 +374,7 @@ spmv_status spmv_partition_colmap(spmv_ctx *ctx, const spmv_csr *A, const int64_
     if (!ctx || !splits || nparts <= 0 || !colmap_out || !slot) { set_error("bad args"); return SPMV_ERR_INVALID_ARG; }
     SPMV_TRY(check_csr(A));
     if (A->n_rows != A->n_cols) { set_error("partition_colmap needs a square matrix"); return SPMV_ERR_INVALID_ARG; }
-    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    SPMV_ON_DEVICE(ctx->device);
     return colmap_impl(ctx, A, splits, nparts, as_stream(stream), colmap_out, slot);
 }
 
@@ -357,7 +387,7 @@ spmv_status spmv_slice_remap_colmap(spmv_ctx *ctx, const spmv_csr *A, const int6
     }
     SPMV_TRY(check_csr(A));
     if (A->n_rows != A->n_cols) { set_error("slice_remap needs a square matrix"); return SPMV_ERR_INVALID_ARG; }
-    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    SPMV_ON_DEVICE(ctx->device);
     return slice_remap_colmap_impl(ctx, A, splits, nparts, part, colmap, as_stream(stream), rp_out, col_out, val_out);
 }
 
@@ -368,7 +398,7 @@ spmv_status spmv_colmap_pack_index(spmv_ctx *ctx, const int32_t *colmap, const i
         return SPMV_ERR_INVALID_ARG;
     }
     if (splits[part + 1] > splits[part] && !idx_out) { set_error("NULL idx_out"); return SPMV_ERR_INVALID_ARG; }
-    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    SPMV_ON_DEVICE(ctx->device);
     return pack_index_impl(ctx, colmap, splits, nparts, part, slot, as_stream(stream), idx_out, count);
 }
 
@@ -381,7 +411,7 @@ spmv_status spmv_slice_split(spmv_ctx *ctx, const spmv_csr *A, const int64_t *sp
     }
     SPMV_TRY(check_csr(A));
     if (A->n_rows != A->n_cols) { set_error("slice_split needs a square matrix"); return SPMV_ERR_INVALID_ARG; }
-    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    SPMV_ON_DEVICE(ctx->device);
     return split_impl(ctx, A, splits, nparts, part, colmap, which, as_stream(stream), rp_out, col_out, val_out, nnz_out);
 }
 
@@ -389,7 +419,7 @@ spmv_status spmv_gather(spmv_ctx *ctx, spmv_dtype dtype, const void *src, const 
                         void *stream) {
     if (!ctx || n < 0 || (n > 0 && (!src || !idx || !dst))) { set_error("bad args"); return SPMV_ERR_INVALID_ARG; }
     if (dtype != SPMV_F32 && dtype != SPMV_F64) { set_error("bad dtype"); return SPMV_ERR_INVALID_ARG; }
-    SPMV_CUDA_TRY(cudaSetDevice(ctx->device));
+    SPMV_ON_DEVICE(ctx->device);
     return gather_impl(ctx, dtype, src, idx, n, dst, as_stream(stream));
 }
 

@@ -578,7 +578,20 @@ spmv_status convert_impl(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, cons
     FeatureSums fs;
     int64_t cusp = 0;
     const bool need_cusp = fmt == SPMV_HYB && o->hyb_width < 0 && o->hyb_rule == 2;
-    SPMV_TRY(feature_pass(ctx, A, s, need_cusp ? 1 : 0, &fs, need_cusp ? &cusp : nullptr));
+    if (o->features) {
+        // the caller's spmv_features result for this matrix: no second pass
+        const spmv_features_t *f = o->features;
+        if (f->n_rows != A->n_rows || f->n_cols != A->n_cols || f->nnz_tot != A->nnz) {
+            set_error("opts.features do not describe this matrix");
+            return SPMV_ERR_INVALID_ARG;
+        }
+        fs = FeatureSums{};
+        fs.len_max = (unsigned long long)f->nnz_max;
+        fs.hyb_coo_ceil = (unsigned long long)f->hyb_coo_nnz;
+        cusp = f->hyb_width_cusp;
+    } else {
+        SPMV_TRY(feature_pass(ctx, A, s, need_cusp ? 1 : 0, &fs, need_cusp ? &cusp : nullptr));
+    }
     if (fs.bad) {
         set_error("matrix is not canonical (flags " + std::to_string(fs.bad) + ")");
         return SPMV_ERR_NOT_CANONICAL;

@@ -2,21 +2,36 @@
 // §IV-A), read per SURVEY A8/A9, plus the canonical-CSR check
 // (A15) that spmv_convert relies on.
 //
-// "Sets 2 and 3 require a scan on the entire matrix, O(nnz)": one
-// streaming pass over col_idx and two over row_ptr, all integer arithmetic with
-// exact 64-bit sums; the fp64 finals are computed on the host from those sums with
-// the fixed formulas of A9, so the result is bit-exact and run-to-run identical.
+// "Sets 2 and 3 require a scan on the entire matrix, O(nnz)": ONE
+// kernel launch reads row_ptr and col_idx once each (vals are never read), with
+// exact 64-bit integer sums; the fp64 finals are computed on the host from those
+// sums with the fixed formulas of A9, so the result is bit-exact and run-to-run
+// identical.  One 112-byte device->host copy returns the result.
 //
-// Block ("continuous nnz chunk") structure is carried by two
-// bitmaps over the nnz positions:
-//   rs[w]   bit l set <=> position 32w+l starts a non-empty row   (F1, row pass)
-//   flag[w] bit l set <=> position 32w+l starts a block           (F2, element pass)
-// A block starts at a row start or wherever col[k] != col[k-1] + 1.  Every row start
-// is a block start, so block sizes are the gaps between consecutive flags (F4) and
-// the number of blocks of row r is F(row_ptr[r+1]) - F(row_ptr[r]) where F(p) counts
-// the flags before p (F3 prefix, F5).
+// Work split (rows + nonzeros balanced, as the merge-path split of A7): the merge
+// of the row STARTS row_ptr[0..n) with the nonzero indices is cut into equal
+// diagonal ranges, one per warp.  A warp finds its two end coordinates with a
+// 32-ary warp-cooperative search (g(i) = row_ptr[i-1] + i, largest i with
+// g(i) <= d) and then walks its range in sub-spans of kSub diagonal items:
+//   phase R  the rows whose start falls in the sub-span (row_ptr read once,
+//            coalesced): row-length sums/min/max, empty rows, HYB overflow, the
+//            A2 row-length histogram, row_ptr validity, and a row-start bitmap of
+//            the sub-span's nonzero positions in shared memory;
+//   phase E  the sub-span's nonzeros, 16 per lane per 512-position chunk (four
+//            16-byte loads): column range/order checks and the block starts
+//            ("continuous nnz chunk": a block starts at a row
+//            start or wherever col[k] != col[k-1] + 1).  Block sizes are the gaps
+//            between consecutive block starts; a row's block count is the number
+//            of block starts between its start and the next row start.  Both are
+//            closed in-lane in position order, with warp scans carrying the last
+//            block start / row start across lanes and chunks.
+// A block or row still open at the end of a warp's range is recorded (WarpRec);
+// the last CTA to finish closes them in one forward pass over the records
+// (at most one open block and one open row per warp), writes the result and
+// resets the accumulators for the next call.  No global bitmaps, no second pass.
 #include <climits>
 #include <cmath>
+#include <mutex>
 #include <vector>
 
 #include "internal.h"
@@ -26,341 +41,667 @@ namespace spmv {
 namespace {
 
 constexpr int kThreads = 256;
-constexpr int kScanChunk = 2048;          // words per local-prefix chunk (256 thr x 8)
-constexpr int kSharedHist = 2048;         // row-length histogram bins kept in smem
+constexpr int kWarps = kThreads / 32;
+constexpr int kCtasPerSm = 2;
+constexpr int kSub = 8192;                      // diagonal items per sub-span
+constexpr int kChunk = 512;                     // nonzero positions per warp chunk (16 per lane)
+constexpr int kBmWords = (kSub + kChunk) / 32;  // row-start bitmap words per warp (+ alignment slack)
+constexpr int kSharedHist = 1024;               // row-length histogram bins kept in shared memory
+constexpr int kRowUnroll = 4;                   // row windows (32 rows) in flight per warp
+constexpr int kRowW = 4;                        // diagonal weight of a row start (a row costs ~4 nonzeros)
 
-enum : unsigned long long {
-    BAD_ROWPTR_ENDS = 1, BAD_ROWPTR_ORDER = 2, BAD_COL_RANGE = 4, BAD_COL_ORDER = 8
-};
+enum : unsigned { BAD_ROWPTR_ENDS = 1, BAD_ROWPTR_ORDER = 2, BAD_COL_RANGE = 4, BAD_COL_ORDER = 8 };
 
 __device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
     return v;
 }
-__device__ __forceinline__ unsigned long long warp_min_u64(unsigned long long v) {
+__device__ __forceinline__ unsigned warp_min_u32(unsigned v) { return __reduce_min_sync(0xffffffffu, v); }
+__device__ __forceinline__ unsigned warp_max_u32(unsigned v) { return __reduce_max_sync(0xffffffffu, v); }
+
+// exclusive prefix sum / max over lanes
+__device__ __forceinline__ unsigned excl_sum(unsigned v, int lane) {
+    unsigned s = v;
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) { unsigned long long t = __shfl_xor_sync(0xffffffffu, v, o); v = t < v ? t : v; }
-    return v;
+    for (int o = 1; o < 32; o <<= 1) {
+        unsigned t = __shfl_up_sync(0xffffffffu, s, o);
+        if (lane >= o) s += t;
+    }
+    return s - v;
 }
-__device__ __forceinline__ unsigned long long warp_max_u64(unsigned long long v) {
+__device__ __forceinline__ int incl_max(int v, int lane) {
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) { unsigned long long t = __shfl_xor_sync(0xffffffffu, v, o); v = t > v ? t : v; }
+    for (int o = 1; o < 32; o <<= 1) {
+        int t = __shfl_up_sync(0xffffffffu, v, o);
+        if (lane >= o && t > v) v = t;
+    }
     return v;
 }
 
-// block-level reduction of (sum..., min, max) into global atomics
-template <int NS>
-__device__ void block_commit(unsigned long long (&sums)[NS], unsigned long long *gsum[NS],
-                             unsigned long long mn, unsigned long long *gmin,
-                             unsigned long long mx, unsigned long long *gmax) {
-    __shared__ unsigned long long s_sum[NS][kThreads / 32];
-    __shared__ unsigned long long s_min[kThreads / 32], s_max[kThreads / 32];
-    int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+// Warp-cooperative 32-ary merge-path search for two diagonals at once (A7 with the
+// row starts as the first list, each row start weighing kRowW items): largest i in
+// [max(0, (d-nnz)/kRowW), min(n, d/kRowW)] with g(i) <= d, g(0) = 0,
+// g(i) = row_ptr[i-1] + kRowW*i.  Every lane returns both results.  On a non-monotone
+// row_ptr the result is still some i in range (the caller only needs termination
+// there; the row walk flags the matrix).
+template <typename IT>
+__device__ __forceinline__ void mp_search2(const IT *__restrict__ rp, int64_t n, int64_t nnz, const int64_t (&d)[2],
+                                           int lane, int64_t (&out)[2]) {
+    int64_t lo[2], hi[2];
 #pragma unroll
-    for (int i = 0; i < NS; ++i) sums[i] = warp_sum_u64(sums[i]);
-    mn = warp_min_u64(mn);
-    mx = warp_max_u64(mx);
-    if (lane == 0) {
-#pragma unroll
-        for (int i = 0; i < NS; ++i) s_sum[i][wid] = sums[i];
-        s_min[wid] = mn;
-        s_max[wid] = mx;
+    for (int t = 0; t < 2; ++t) {
+        lo[t] = d[t] - nnz > 0 ? (d[t] - nnz) / kRowW : 0;
+        hi[t] = d[t] / kRowW < n ? d[t] / kRowW : n;
+        if (hi[t] < lo[t]) hi[t] = lo[t];
     }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        for (int w = 1; w < kThreads / 32; ++w) {
+    while (hi[0] > lo[0] || hi[1] > lo[1]) {
+        int64_t q[2];
+        bool ok[2];
 #pragma unroll
-            for (int i = 0; i < NS; ++i) s_sum[i][0] += s_sum[i][w];
-            s_min[0] = s_min[w] < s_min[0] ? s_min[w] : s_min[0];
-            s_max[0] = s_max[w] > s_max[0] ? s_max[w] : s_max[0];
+        for (int t = 0; t < 2; ++t) {
+            const int64_t len = hi[t] - lo[t];
+            q[t] = lo[t] + 1 + ((int64_t)lane * len) / 32;
+            ok[t] = true;
+            if (len > 0) ok[t] = (int64_t)__ldg(rp + q[t] - 1) + kRowW * q[t] <= d[t];
         }
 #pragma unroll
-        for (int i = 0; i < NS; ++i)
-            if (gsum[i] && s_sum[i][0]) atomicAdd(gsum[i], s_sum[i][0]);
-        if (gmin) atomicMin(gmin, s_min[0]);
-        if (gmax) atomicMax(gmax, s_max[0]);
+        for (int t = 0; t < 2; ++t) {
+            const unsigned m = __ballot_sync(0xffffffffu, ok[t]);
+            const int j = m == 0xffffffffu ? 32 : __ffs(~m) - 1;     // leading lanes with g(q) <= d
+            const int64_t qa = __shfl_sync(0xffffffffu, q[t], j > 0 ? j - 1 : 0);
+            const int64_t qb = __shfl_sync(0xffffffffu, q[t], j < 32 ? j : 31);
+            if (hi[t] > lo[t]) {
+                if (j == 0) hi[t] = lo[t];
+                else if (j == 32) lo[t] = qa;
+                else { lo[t] = qa; hi[t] = qb - 1; }
+            }
+        }
     }
+    out[0] = lo[0];
+    out[1] = lo[1];
 }
 
-// F1: row pass -- row lengths (sum len^2, min, max, empty rows, HYB overflow),
-// row_ptr validity, row-start bitmap, row-length histogram for the A2 "cusp" rule.
+}  // namespace
+
+// Per-warp record for the cross-warp fix-up (one block and one row may stay open).
+struct WarpRec {
+    long long first_flag;        // first block start in the warp's range (-1: none)
+    long long last_flag;         // last block start (-1: none)
+    unsigned long long nflags;   // block starts in the range
+    unsigned long long head_nb;  // block starts before the first row start of the range
+    long long has_rs;            // a row starts inside the range
+    unsigned long long open_tail;// block starts from the start of the row still open at the end
+    long long has_open;          // a row starting in the range ends past it
+};
+
+// Device state of the feature pass, owned by the ctx: atomically accumulated sums
+// (reset by the last CTA of every launch), the done counter and the result.
+struct FeatureState {
+    FeatureSums acc;
+    unsigned long long done;
+    FeatureSums result;
+    long long cusp;
+};
+
+namespace {
+
+// records and histogram are written by other CTAs: read them at L2 (no stale L1 lines)
+__device__ __forceinline__ WarpRec load_rec(const WarpRec *p) {
+    WarpRec r;
+    r.first_flag = __ldcg(&p->first_flag);
+    r.last_flag = __ldcg(&p->last_flag);
+    r.nflags = __ldcg(&p->nflags);
+    r.head_nb = __ldcg(&p->head_nb);
+    r.has_rs = __ldcg(&p->has_rs);
+    r.open_tail = __ldcg(&p->open_tail);
+    r.has_open = __ldcg(&p->has_open);
+    return r;
+}
+
+__device__ __forceinline__ void init_sums(FeatureSums &s) {
+    s.bad = 0; s.n_empty = 0; s.sum_len2 = 0; s.len_min = ULLONG_MAX; s.len_max = 0; s.hyb_coo_ceil = 0;
+    s.nb_tot = 0; s.sum_nb2 = 0; s.nb_min = ULLONG_MAX; s.nb_max = 0; s.sum_bs2 = 0;
+    s.bs_min = ULLONG_MAX; s.bs_max = 0;
+}
+
 template <typename IT>
-__global__ void __launch_bounds__(kThreads)
-k_rows(const IT *__restrict__ rp, int64_t n_rows, int64_t nnz, int64_t kh,
-       unsigned *__restrict__ rs_bits, unsigned long long *__restrict__ hist, int64_t hist_bins,
-       FeatureSums *out) {
+__global__ void __launch_bounds__(kThreads, kCtasPerSm)
+k_features(const IT *__restrict__ rp, const int *__restrict__ col, int64_t n, int64_t nnz, int64_t n_cols,
+           int64_t kh, int64_t per_warp, WarpRec *__restrict__ recs, unsigned long long *__restrict__ hist,
+           int64_t hist_bins, FeatureState *st) {
+    using P = IT;                       // nonzero positions: 32-bit arithmetic for int32 row_ptr
+    constexpr P kNone = sizeof(P) == 4 ? (P)INT_MIN : (P)LLONG_MIN;
+    // per warp: the sub-span's row-start bits, its block-start bits (flags) and the
+    // exclusive prefix of flag popcounts per word
+    __shared__ unsigned s_bm[kWarps][kBmWords];
+    __shared__ unsigned s_fl[kWarps][kBmWords];
+    __shared__ unsigned s_pf[kWarps][kBmWords];
     __shared__ unsigned s_hist[kSharedHist];
+    __shared__ bool s_last;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const bool use_hist = hist != nullptr;
     const int sh_bins = hist_bins < kSharedHist ? (int)hist_bins : kSharedHist;
     if (use_hist)
-        for (int i = threadIdx.x; i < sh_bins; i += blockDim.x) s_hist[i] = 0;
-    __syncthreads();
-    unsigned long long bad = 0, len2 = 0, empty = 0, over = 0;
-    unsigned long long mn = ULLONG_MAX, mx = 0;
-    if (blockIdx.x == 0 && threadIdx.x == 0)
-        if ((int64_t)rp[0] != 0 || (int64_t)rp[n_rows] != nnz) bad |= BAD_ROWPTR_ENDS;
-    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n_rows;
-         r += (int64_t)gridDim.x * blockDim.x) {
-        int64_t a = rp[r], b = rp[r + 1];
-        int64_t len = b - a;
-        if (len < 0 || a < 0 || b > nnz) { bad |= BAD_ROWPTR_ORDER; len = 0; }
-        unsigned long long ul = (unsigned long long)len;
-        len2 += ul * ul;
-        mn = ul < mn ? ul : mn;
-        mx = ul > mx ? ul : mx;
-        empty += (len == 0);
-        over += len > kh ? (unsigned long long)(len - kh) : 0ull;
-        if (len > 0) atomicOr(&rs_bits[a >> 5], 1u << (a & 31));
-        if (use_hist) {
-            // rows of a warp mostly share a length bin: one shared atomic per distinct bin
-            const int64_t bin = len < hist_bins - 1 ? len : hist_bins - 1;
-            const unsigned active = __activemask();
-            const unsigned same = __match_any_sync(active, (unsigned long long)bin);
-            if ((threadIdx.x & 31) == __ffs(same) - 1) {
-                if (bin < sh_bins) atomicAdd(&s_hist[bin], (unsigned)__popc(same));
-                else atomicAdd(&hist[bin], (unsigned long long)__popc(same));
-            }
-        }
-    }
-    if (bad) atomicOr(&out->bad, bad);
-    unsigned long long sums[3] = {len2, empty, over};
-    unsigned long long *g[3] = {&out->sum_len2, &out->n_empty, &out->hyb_coo_ceil};
-    block_commit<3>(sums, g, mn, &out->len_min, mx, &out->len_max);
-    if (use_hist) {
-        __syncthreads();
-        for (int i = threadIdx.x; i < sh_bins; i += blockDim.x)
-            if (s_hist[i]) atomicAdd(&hist[i], (unsigned long long)s_hist[i]);
-    }
-}
-
-// F2: element pass -- column validity/order and the block-start bitmap.  A warp
-// handles a chunk of 512 positions (16 words) per iteration: lane l loads its 16
-// consecutive elements with four 16-byte loads, derives 16 flag bits, and lane pairs
-// merge their half-words into the chunk's flag words.
-constexpr int kLaneElems = 16;
-constexpr int kChunkWords = kLaneElems;      // 32 lanes x 16 elements = 16 words
-
-__global__ void __launch_bounds__(kThreads)
-k_flags(const int *__restrict__ col, int64_t nnz, int64_t n_cols, int64_t n_words,
-        const unsigned *__restrict__ rs_bits, unsigned *__restrict__ flag_bits, FeatureSums *out) {
-    const int lane = threadIdx.x & 31;
-    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t n_warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+        for (int i = threadIdx.x; i < sh_bins; i += kThreads) s_hist[i] = 0;
+    unsigned *bm = s_bm[wid];
+    unsigned *fl = s_fl[wid];
+    unsigned *pf = s_pf[wid];
     const uint64_t pol = policy_evict_first();
+    constexpr int kCap = kBmWords * 32;
+    const bool col_aligned = (reinterpret_cast<uintptr_t>(col) & 15) == 0;
+
+    const int64_t items = (int64_t)kRowW * n + nnz;
+    const int64_t W = (int64_t)gridDim.x * kWarps;
+    const int64_t w = (int64_t)blockIdx.x * kWarps + wid;
+    int64_t dd[2], ii[2];
+    dd[0] = w * per_warp < items ? w * per_warp : items;
+    dd[1] = dd[0] + per_warp < items ? dd[0] + per_warp : items;
+    mp_search2(rp, n, nnz, dd, lane, ii);
+    const int64_t d0 = dd[0], d1 = dd[1];
+    const int64_t i0 = w == 0 ? 0 : ii[0];
+    const int64_t i1 = w == W - 1 ? n : ii[1];
+    auto clampk = [&](int64_t k) { return (P)(k < 0 ? 0 : (k > nnz ? nnz : k)); };
+    // coordinate (i, k): i row starts and k = min(d - kRowW*i, row_ptr[i]) nonzeros consumed
+    const int64_t rpi0 = (int64_t)__ldg(rp + i0), rpi1 = (int64_t)__ldg(rp + i1);
+    const P k0 = w == 0 ? (P)0 : clampk(d0 - kRowW * i0 < rpi0 ? d0 - kRowW * i0 : rpi0);
+    P k1 = w == W - 1 ? (P)nnz : clampk(d1 - kRowW * i1 < rpi1 ? d1 - kRowW * i1 : rpi1);
+    if (k1 < k0) k1 = k0;
+
     unsigned bad = 0;
-    for (int64_t wb = warp * kChunkWords; wb < n_words; wb += n_warps * kChunkWords) {
-        const int64_t k0 = wb * 32 + (int64_t)lane * kLaneElems;      // this lane's first position
-        int c[kLaneElems];
-        if (k0 + kLaneElems <= nnz && ((uintptr_t)(col + k0) & 15) == 0) {
+    if (w == 0 && lane == 0)
+        if ((int64_t)rp[0] != 0 || (int64_t)rp[n] != nnz) bad |= BAD_ROWPTR_ENDS;
+
+    // per-lane accumulators
+    unsigned long long len2 = 0, over = 0, nb2 = 0, sz2 = 0;
+    unsigned len_mn = UINT_MAX, len_mx = 0, n_empty = 0, nb_mn = UINT_MAX, nb_mx = 0, sz_mn = UINT_MAX, sz_mx = 0;
+    // warp-uniform state
+    P c_lastflag = kNone;           // position of the last block start so far (kNone: none)
+    unsigned c_F = 0;               // block starts so far in the warp's range
+    long long head_nb = -1;         // flags before the first row start of the range (-1: none yet)
+    long long c_Frs = -1;           // flags before the last row start so far (-1: none yet)
+    P my_first_flag = kNone;        // set by the single lane that meets the range's first block start
+
+    // the range's first nonzero starts a row owned (row-walk-wise) by the previous warp:
+    // its row-start bit is set here, so its block count is this warp's
+    bool pending_rs = i0 > 0 && k0 < k1 && (int64_t)__ldg(rp + i0 - 1) == (int64_t)k0;
+
+    int64_t r = i0, dcur = d0;
+    P kcur = k0;
+    while (true) {
+        const int64_t dsub = dcur + kSub < d1 ? dcur + kSub : d1;
+        const bool last = dsub == d1;
+        const P base = kcur & ~(P)15;
+        const int kc_rel = (int)(kcur - base);
+        int prevc = 0;                  // col[kcur-1]: latency hidden by phase R1
+        if (kcur > 0 && kcur < k1) prevc = __ldg(col + kcur - 1);
+        for (int i = lane; i < kBmWords; i += 32) { bm[i] = 0u; fl[i] = 0u; }
+        __syncwarp();
+        if (pending_rs && lane == 0) atomicOr(&bm[kc_rel >> 5], 1u << (kc_rel & 31));
+
+        // ---- R1: rows r with g(r+1) = row_ptr[r] + kRowW*(r+1) <= dsub (every row < i1 when
+        //      last), taken strictly in order: lengths (sums, min/max, empty, HYB overflow,
+        //      histogram), row_ptr validity, and row-start bits of their start positions.
+        //      Relative form: (row_ptr[r] - base) + kRowW*(r - r_start) <= lim.
+        const int64_t r_start = r;
+        const int64_t lim64 = dsub - kRowW * (r_start + 1) - (int64_t)base;
+        const int lim = last ? INT_MAX : (int)(lim64 < INT_MIN ? INT_MIN : (lim64 > INT_MAX ? INT_MAX : lim64));
+        const int64_t jmax64 = i1 - r_start;
+        const int jmax = (int)(jmax64 < INT_MAX - 1024 ? jmax64 : INT_MAX - 1024);
+        while (r < i1) {
+            IT a[kRowUnroll + 1];
 #pragma unroll
-            for (int q = 0; q < kLaneElems / 4; ++q) {
-                const int4 v = ld_hint(reinterpret_cast<const int4 *>(col + k0) + q, pol);
-                c[4 * q] = v.x; c[4 * q + 1] = v.y; c[4 * q + 2] = v.z; c[4 * q + 3] = v.w;
+            for (int u = 0; u < kRowUnroll; ++u) {
+                const int64_t rr = r + u * 32 + lane;
+                a[u] = __ldg(rp + (rr < n ? rr : n));
             }
-        } else {
+            a[kRowUnroll] = __ldg(rp + (r + 32 * kRowUnroll < n ? r + 32 * kRowUnroll : n));
+            const int j0 = (int)(r - r_start);
+            int taken = 0;
+            bool stop = false;
 #pragma unroll
-            for (int e = 0; e < kLaneElems; ++e) c[e] = k0 + e < nnz ? col[k0 + e] : 0;
-        }
-        const unsigned rw = (wb + (lane >> 1) < n_words) ? rs_bits[wb + (lane >> 1)] : 0u;
-        const unsigned rs16 = (rw >> ((lane & 1) * 16)) & 0xFFFFu;
-        int prev = __shfl_up_sync(0xffffffffu, c[kLaneElems - 1], 1);
-        if (lane == 0) prev = (k0 > 0 && k0 < nnz) ? col[k0 - 1] : 0;
-        unsigned f16 = 0;
-#pragma unroll
-        for (int e = 0; e < kLaneElems; ++e) {
-            const int64_t k = k0 + e;
-            const bool valid = k < nnz;
-            const int pv = e == 0 ? prev : c[e - 1];
-            const bool rowstart = (rs16 >> e) & 1u;
-            const bool flag = valid && (rowstart || k == 0 || (int64_t)c[e] != (int64_t)pv + 1);
-            if (valid && (c[e] < 0 || (int64_t)c[e] >= n_cols)) bad |= BAD_COL_RANGE;
-            if (valid && k > 0 && !rowstart && c[e] <= pv) bad |= BAD_COL_ORDER;
-            if (valid && k == 0 && !rowstart) bad |= BAD_ROWPTR_ORDER;
-            f16 |= (unsigned)flag << e;
-        }
-        const unsigned hi = __shfl_down_sync(0xffffffffu, f16, 1);
-        if (!(lane & 1) && wb + (lane >> 1) < n_words) flag_bits[wb + (lane >> 1)] = f16 | (hi << 16);
-    }
-    bad = __reduce_or_sync(0xffffffffu, bad);
-    if (lane == 0 && bad) atomicOr(&out->bad, (unsigned long long)bad);
-}
-
-// F3a: per-chunk exclusive prefix of flag popcounts (kScanChunk words per block).
-__global__ void __launch_bounds__(kThreads)
-k_scan_local(const unsigned *__restrict__ flag_bits, int64_t n_words, unsigned *__restrict__ local,
-             unsigned long long *__restrict__ totals) {
-    __shared__ unsigned s_warp[kThreads / 32];
-    const int64_t base = (int64_t)blockIdx.x * kScanChunk;
-    constexpr int per = kScanChunk / kThreads;   // 8 consecutive words per thread
-    unsigned cnt[per];
-    unsigned tsum = 0;
-#pragma unroll
-    for (int i = 0; i < per; ++i) {
-        int64_t w = base + threadIdx.x * per + i;
-        cnt[i] = w < n_words ? __popc(flag_bits[w]) : 0u;
-        tsum += cnt[i];
-    }
-    // block exclusive scan of tsum
-    int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    unsigned incl = tsum;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        unsigned t = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += t;
-    }
-    if (lane == 31) s_warp[wid] = incl;
-    __syncthreads();
-    unsigned woff = 0;
-    for (int i = 0; i < wid; ++i) woff += s_warp[i];
-    unsigned run = woff + incl - tsum;
-#pragma unroll
-    for (int i = 0; i < per; ++i) {
-        int64_t w = base + threadIdx.x * per + i;
-        if (w < n_words) local[w] = run;
-        run += cnt[i];
-    }
-    if (threadIdx.x == kThreads - 1) totals[blockIdx.x] = run;
-}
-
-// F3b: exclusive scan of the chunk totals (one block, sequential over tiles of 256).
-__global__ void __launch_bounds__(kThreads)
-k_scan_totals(unsigned long long *totals, int64_t n) {
-    __shared__ unsigned long long s_warp[kThreads / 32];
-    __shared__ unsigned long long s_carry;
-    if (threadIdx.x == 0) s_carry = 0;
-    __syncthreads();
-    int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    for (int64_t base = 0; base < n; base += kThreads) {
-        int64_t i = base + threadIdx.x;
-        unsigned long long v = i < n ? totals[i] : 0ull, incl = v;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            unsigned long long t = __shfl_up_sync(0xffffffffu, incl, o);
-            if (lane >= o) incl += t;
-        }
-        if (lane == 31) s_warp[wid] = incl;
-        __syncthreads();
-        unsigned long long woff = 0;
-        for (int k = 0; k < wid; ++k) woff += s_warp[k];
-        unsigned long long carry = s_carry;
-        if (i < n) totals[i] = carry + woff + incl - v;
-        __syncthreads();
-        if (threadIdx.x == kThreads - 1) s_carry = carry + woff + incl;
-        __syncthreads();
-    }
-}
-
-// F4: block sizes = gaps between consecutive block starts.  A warp takes 256 words
-// (8192 positions) per iteration, lane l the 8 words [8l, 8l+8) loaded as two 16-byte
-// vectors; a lane walks its flags in order (gap to the previous flag = one block), the
-// block left open at the lane end closes at the first flag of a later lane (suffix
-// minimum over lanes) or, past the chunk, at the next flagged word (forward scan).
-constexpr int kLaneWords = 8;
-
-__global__ void __launch_bounds__(kThreads)
-k_block_sizes(const unsigned *__restrict__ flag_bits, int64_t n_words, int64_t nnz, FeatureSums *out) {
-    const int lane = threadIdx.x & 31;
-    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t n_warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    constexpr int64_t CW = 32 * kLaneWords;
-    unsigned long long nb = 0, sz2 = 0, mn = ULLONG_MAX, mx = 0;
-    auto take = [&](unsigned long long sz) {
-        nb += 1;
-        sz2 += sz * sz;
-        mn = sz < mn ? sz : mn;
-        mx = sz > mx ? sz : mx;
-    };
-    for (int64_t wb = warp * CW; wb < n_words; wb += n_warps * CW) {
-        const int64_t w0 = wb + (int64_t)lane * kLaneWords;
-        unsigned fw[kLaneWords];
-        // flag_bits is padded to a multiple of CW words (zeros): vector loads stay inside
-        const uint4 a = *reinterpret_cast<const uint4 *>(flag_bits + w0);
-        const uint4 b = *reinterpret_cast<const uint4 *>(flag_bits + w0 + 4);
-        fw[0] = a.x; fw[1] = a.y; fw[2] = a.z; fw[3] = a.w; fw[4] = b.x; fw[5] = b.y; fw[6] = b.z; fw[7] = b.w;
-        int64_t first = -1, last = -1;
-#pragma unroll
-        for (int q = 0; q < kLaneWords; ++q) {
-            unsigned w = fw[q];
-            while (w) {
-                const int64_t p = (w0 + q) * 32 + (__ffs(w) - 1);
-                w &= w - 1;
-                if (last >= 0) take((unsigned long long)(p - last));
-                else first = p;
-                last = p;
+            for (int u = 0; u < kRowUnroll; ++u) {
+                const int j = j0 + u * 32 + lane;
+                const P arel = (P)(a[u] - base);
+                const bool want = j < jmax && (last || arel + (P)(kRowW * j) <= (P)lim);
+                const unsigned wm = __ballot_sync(0xffffffffu, want);
+                const int plen = stop ? 0 : (wm == 0xffffffffu ? 32 : __ffs(~wm) - 1);
+                const bool inr = lane < plen;
+                const P nx = __shfl_down_sync(0xffffffffu, a[u], 1);
+                const P nw = u + 1 < kRowUnroll ? __shfl_sync(0xffffffffu, a[u + 1 < kRowUnroll ? u + 1 : u], 0)
+                                                : a[kRowUnroll];       // first row of the next window
+                const P bb = lane == 31 ? nw : nx;
+                P len = bb - a[u];
+                if (inr) {
+                    if (arel >= (P)kc_rel && arel < (P)kCap) atomicOr(&bm[(int)arel >> 5], 1u << ((int)arel & 31));
+                    if (len < 0 || a[u] < 0 || (int64_t)bb > nnz) { bad |= BAD_ROWPTR_ORDER; len = 0; }
+                    const unsigned ul = (unsigned)len;
+                    len2 += (unsigned long long)ul * ul;
+                    len_mn = min(len_mn, ul);
+                    len_mx = max(len_mx, ul);
+                    n_empty += len == 0;
+                    over += (int64_t)len > kh ? (unsigned long long)((int64_t)len - kh) : 0ull;
+                }
+                if (use_hist) {                                      // empty rows: n_empty (bin 0)
+                    const bool hb = inr && len > 0;
+                    const unsigned bin = hb ? (unsigned)((int64_t)len < hist_bins - 1 ? (int64_t)len : hist_bins - 1) : 0u;
+                    const unsigned hm = __ballot_sync(0xffffffffu, hb);
+                    if (hm) {
+                        const int lead = __ffs(hm) - 1;
+                        const unsigned b0 = __shfl_sync(0xffffffffu, bin, lead);
+                        if (__all_sync(0xffffffffu, !hb || bin == b0)) {  // one length bin for the window
+                            if (lane == lead) {
+                                if ((int)b0 < sh_bins) atomicAdd(&s_hist[b0], (unsigned)__popc(hm));
+                                else atomicAdd(&hist[b0], (unsigned long long)__popc(hm));
+                            }
+                        } else if (hb) {
+                            if ((int)bin < sh_bins) atomicAdd(&s_hist[bin], 1u);
+                            else atomicAdd(&hist[bin], 1ull);
+                        }
+                    }
+                }
+                taken += plen;
+                if (plen < 32) stop = true;
             }
+            r += taken;
+            if (stop) break;
         }
-        // first flag strictly after this lane: suffix minimum of `first` over later lanes
-        int64_t nxt = first >= 0 ? first : INT64_MAX;
+        const int64_t r_end = r;
+        P knext = k1;
+        if (!last) {
+            const int64_t rpe = (int64_t)__ldg(rp + (r_end < n ? r_end : n));
+            const int64_t kk = dsub - kRowW * r_end;
+            knext = clampk(kk < rpe ? kk : rpe);
+            if (knext < kcur) knext = kcur;
+            if (knext > k1) knext = k1;
+        }
+        const int kn_rel = (int)(knext - base);
+        __syncwarp();
+        // a row start exactly at knext belongs to the next sub-span's first position
+        const bool pending_next = knext < k1 && kn_rel < kCap && ((bm[kn_rel >> 5] >> (kn_rel & 31)) & 1u);
+        __syncwarp();
+
+        // ---- E: nonzeros [kcur, knext), 16 per lane per 512-position chunk from `base`:
+        //      checks, block starts (written over the row-start bits), block sizes
+        const unsigned F_sub = c_F;
+        // a lane's 16 columns of the chunk at relative position cr (next chunk prefetched)
+        auto load16 = [&](int cr, int (&v)[16]) {
+            const P q0 = base + (P)(cr + lane * 16);
+            if (col_aligned && (int64_t)q0 + 16 <= nnz) {
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int64_t v = __shfl_down_sync(0xffffffffu, nxt, o);
-            if (lane + o < 32 && v < nxt) nxt = v;
-        }
-        int64_t after = __shfl_down_sync(0xffffffffu, nxt, 1);
-        if (lane == 31) after = INT64_MAX;
-        // past the chunk: the next flagged word (warp-cooperative forward scan, rare)
-        const bool need = __any_sync(0xffffffffu, last >= 0 && after == INT64_MAX);
-        if (need) {
-            int64_t beyond = nnz;
-            for (int64_t base = wb + CW; base < n_words; base += 32) {
-                const unsigned v = base + lane < n_words ? flag_bits[base + lane] : 0u;
-                const unsigned bm = __ballot_sync(0xffffffffu, v != 0u);
-                if (bm) {
-                    const int src = __ffs(bm) - 1;
-                    const unsigned fv = __shfl_sync(0xffffffffu, v, src);
-                    beyond = (base + src) * 32 + (__ffs(fv) - 1);
-                    break;
+                for (int q = 0; q < 4; ++q) {
+                    const int4 t = ld_hint(reinterpret_cast<const int4 *>(col + q0) + q, pol);
+                    v[4 * q] = t.x; v[4 * q + 1] = t.y; v[4 * q + 2] = t.z; v[4 * q + 3] = t.w;
+                }
+            } else {
+#pragma unroll
+                for (int e = 0; e < 16; ++e) v[e] = (int64_t)q0 + e < nnz ? __ldg(col + q0 + e) : 0;
+            }
+        };
+        int cn[16];
+        if (kn_rel > 0) load16(0, cn);
+        for (int cr = 0; cr < kn_rel; cr += kChunk) {
+            const int off = cr + lane * 16;                          // relative position of the lane's first
+            const P p0 = base + (P)off;
+            int c[16];
+#pragma unroll
+            for (int e = 0; e < 16; ++e) c[e] = cn[e];
+            if (cr + kChunk < kn_rel) load16(cr + kChunk, cn);
+            const unsigned rs16 = (bm[off >> 5] >> (off & 31)) & 0xFFFFu;
+            int pv = __shfl_up_sync(0xffffffffu, c[15], 1);
+            if (lane == 0) pv = prevc;
+            prevc = __shfl_sync(0xffffffffu, c[15], 31);
+            const int lo_e = min(max(kc_rel - off, 0), 16);
+            const int hi_e = min(max(kn_rel - off, 0), 16);
+            const unsigned v16 = hi_e > lo_e ? (((1u << hi_e) - 1u) & ~((1u << lo_e) - 1u)) : 0u;
+            unsigned fr = 0, ob = 0, cmax = 0;
+#pragma unroll
+            for (int e = 0; e < 16; ++e) {
+                const int u = c[e] - (e == 0 ? pv : c[e - 1]) - 1;   // 0: the next column
+                fr |= (unsigned)(u != 0) << e;                        // a block starts
+                ob |= ((unsigned)u >> 31) << e;                      // not increasing: only at a row start
+                cmax = max(cmax, (unsigned)c[e]);
+            }
+            const unsigned rsv = rs16 & v16;
+            const unsigned f16 = (fr | rsv) & v16;
+            if (ob & ~rsv & v16) bad |= BAD_COL_ORDER;
+            if (v16 && (unsigned long long)cmax >= (unsigned long long)n_cols) bad |= BAD_COL_RANGE;
+            const unsigned f_up = __shfl_up_sync(0xffffffffu, f16, 1);
+            {
+                const unsigned hi = __shfl_down_sync(0xffffffffu, f16, 1);
+                if (!(lane & 1)) fl[off >> 5] = f16 | (hi << 16);
+            }
+            // block sizes = gaps between consecutive block starts.  A start whose previous
+            // position is a start closes a block of size 1 (bit test, no loop); the others
+            // (block >= 2, or the range's first start) walk back to the previous start.
+            unsigned fprev = (f16 << 1) | (f_up >> 15);
+            if (lane == 0) {
+                const int q0 = max(off, kc_rel);                     // first valid position of lane 0
+                fprev = (f16 << 1) | ((c_lastflag == base + (P)q0 - 1) ? 1u << (q0 - off) : 0u);
+            }
+            const unsigned s1 = f16 & fprev;
+            const unsigned c1 = __popc(s1);
+            sz2 += c1;
+            if (c1) { sz_mn = 1u; sz_mx = max(sz_mx, 1u); }
+            const int rel_last = f16 ? off + 31 - __clz(f16) : INT_MIN;
+            const int incl = incl_max(rel_last, lane);
+            const int before = __shfl_up_sync(0xffffffffu, incl, 1);
+            int lastf_in;                                            // sub-span-relative previous start
+            if (lane > 0 && before != INT_MIN) lastf_in = before;
+            else if (c_lastflag != kNone) {
+                const int64_t dl = (int64_t)c_lastflag - (int64_t)base;
+                lastf_in = (int)(dl > (int64_t)INT_MIN + 1 ? dl : (int64_t)INT_MIN + 1);
+            } else lastf_in = INT_MIN;
+            unsigned rem = f16 & ~s1;
+            while (rem) {
+                const int e = __ffs(rem) - 1;
+                rem &= rem - 1u;
+                const unsigned below = f16 & ((1u << e) - 1u);
+                const int pf_ = below ? off + 31 - __clz(below) : lastf_in;
+                if (pf_ == INT_MIN) {
+                    my_first_flag = p0 + (P)e;
+                } else {
+                    const unsigned sz = (unsigned)(off + e - pf_);
+                    sz2 += (unsigned long long)sz * sz;
+                    sz_mn = min(sz_mn, sz);
+                    sz_mx = max(sz_mx, sz);
                 }
             }
-            if (after == INT64_MAX) after = beyond;
+            const int last_in_chunk = __shfl_sync(0xffffffffu, incl, 31);
+            if (last_in_chunk != INT_MIN) c_lastflag = base + (P)last_in_chunk;
+            c_F += __reduce_add_sync(0xffffffffu, (unsigned)__popc(f16));
         }
-        if (last >= 0) take((unsigned long long)(after - last));
+        __syncwarp();
+
+        // ---- P: exclusive prefix of the flag popcounts per bitmap word (words up to knext)
+        {
+            const int wk = kn_rel >> 5;
+            constexpr int per = (kBmWords + 31) / 32;
+            unsigned cnt[per], tot = 0;
+#pragma unroll
+            for (int j = 0; j < per; ++j) {
+                const int wi = lane * per + j;
+                cnt[j] = (wi < kBmWords && wi <= wk) ? __popc(fl[wi]) : 0u;
+                tot += cnt[j];
+            }
+            unsigned run = excl_sum(tot, lane);
+#pragma unroll
+            for (int j = 0; j < per; ++j) {
+                const int wi = lane * per + j;
+                if (wi < kBmWords) pf[wi] = run;
+                run += cnt[j];
+            }
+        }
+        __syncwarp();
+        // ---- B: blocks per row.  A (non-empty) row's block count is the number of block
+        //      starts from its start to the next row start, F(next) - F(start) with F(p) =
+        //      flags before p.  The sub-span's T row starts (valid positions) are dealt to
+        //      the lanes in order, T/32 each: lane l closes rows [lT/32, (l+1)T/32).
+        {
+            constexpr int per = (kBmWords + 31) / 32;
+            const int wk = kn_rel >> 5;
+            auto vmask = [&](int wi) -> unsigned {                   // valid positions [kc_rel, kn_rel)
+                const int lo = kc_rel - 32 * wi, hi = kn_rel - 32 * wi;
+                return (hi >= 32 ? 0xffffffffu : (hi <= 0 ? 0u : (1u << hi) - 1u)) &
+                       (lo <= 0 ? 0xffffffffu : (lo >= 32 ? 0u : ~((1u << lo) - 1u)));
+            };
+            unsigned cnt = 0;
+#pragma unroll
+            for (int j = 0; j < per; ++j) {
+                const int wi = lane * per + j;
+                if (wi < kBmWords && wi <= wk) cnt += __popc(bm[wi] & vmask(wi));
+            }
+            const unsigned ex = excl_sum(cnt, lane);
+            const unsigned T = __shfl_sync(0xffffffffu, ex + cnt, 31);
+            if (T > 0) {
+                const unsigned s0 = (unsigned)(((unsigned long long)lane * T) >> 5);
+                const unsigned s1 = (unsigned)(((unsigned long long)(lane + 1) * T) >> 5);
+                // owner of row start s0: the last lane o with ex_o <= s0
+                int o = 0;
+#pragma unroll
+                for (int step = 16; step > 0; step >>= 1) {
+                    const unsigned e2 = __shfl_sync(0xffffffffu, ex, o + step);
+                    if (e2 <= s0) o += step;
+                }
+                const unsigned exo = __shfl_sync(0xffffffffu, ex, o);
+                long long F_first = -1, F_last = -1;
+                if (s1 > s0) {
+                    // the (s0 - ex_o)-th row start inside lane o's words
+                    unsigned skip = s0 - exo;
+                    int wi = o * per;
+                    unsigned m = bm[wi] & vmask(wi);
+                    while (__popc(m) <= skip) { skip -= __popc(m); ++wi; m = bm[wi] & vmask(wi); }
+                    for (; skip; --skip) m &= m - 1u;
+                    for (unsigned k = s0; k < s1; ++k) {
+                        const int b = __ffs(m) - 1;
+                        const long long Fp = (long long)(F_sub + pf[wi] + __popc(fl[wi] & ((1u << b) - 1u)));
+                        if (F_last >= 0) {
+                            const unsigned nb = (unsigned)(Fp - F_last);
+                            nb2 += (unsigned long long)nb * nb;
+                            nb_mn = min(nb_mn, nb);
+                            nb_mx = max(nb_mx, nb);
+                        } else {
+                            F_first = Fp;
+                        }
+                        F_last = Fp;
+                        m &= m - 1u;
+                        if (k + 1 < s1)
+                            while (!m) { ++wi; m = bm[wi] & vmask(wi); }
+                    }
+                }
+                // the last row of a lane ends at the next working lane's first row start
+                const unsigned workm = __ballot_sync(0xffffffffu, s1 > s0);
+                const unsigned later = workm & ~((2u << lane) - 1u);
+                const long long F_next = __shfl_sync(0xffffffffu, F_first, later ? __ffs(later) - 1 : 0);
+                if (s1 > s0 && later) {
+                    const unsigned nb = (unsigned)(F_next - F_last);
+                    nb2 += (unsigned long long)nb * nb;
+                    nb_mn = min(nb_mn, nb);
+                    nb_mx = max(nb_mx, nb);
+                }
+                // the first row start closes the row left open before the sub-span
+                const int firstw = __ffs(workm) - 1, lastw = 31 - __clz(workm);
+                const long long F0 = __shfl_sync(0xffffffffu, F_first, firstw);
+                const long long FL = __shfl_sync(0xffffffffu, F_last, lastw);
+                if (c_Frs >= 0) {
+                    if (lane == 0) {
+                        const unsigned nb = (unsigned)(F0 - c_Frs);
+                        nb2 += (unsigned long long)nb * nb;
+                        nb_mn = min(nb_mn, nb);
+                        nb_mx = max(nb_mx, nb);
+                    }
+                } else if (head_nb < 0) {
+                    head_nb = F0;                                     // the range's first row start
+                }
+                c_Frs = FL;
+            }
+        }
+        __syncwarp();
+        pending_rs = pending_next;
+        kcur = knext;
+        dcur = dsub;
+        if (last) break;
     }
-    unsigned long long sums[2] = {nb, sz2};
-    unsigned long long *g[2] = {&out->nb_tot, &out->sum_bs2};
-    block_commit<2>(sums, g, mn, &out->bs_min, mx, &out->bs_max);
-}
 
-__device__ __forceinline__ unsigned long long flags_before(int64_t p, int64_t n_words,
-                                                           const unsigned *__restrict__ flag_bits,
-                                                           const unsigned *__restrict__ local,
-                                                           const unsigned long long *__restrict__ totals,
-                                                           unsigned long long total_flags) {
-    int64_t w = p >> 5;
-    if (w >= n_words) return total_flags;
-    unsigned m = (p & 31) ? (flag_bits[w] & ((1u << (p & 31)) - 1u)) : 0u;
-    return totals[w / kScanChunk] + local[w] + __popc(m);
-}
-
-// F5: blocks per row (nnzb_*), over all rows including empty ones (A8).
-template <typename IT>
-__global__ void __launch_bounds__(kThreads)
-k_row_blocks(const IT *__restrict__ rp, int64_t n_rows, int64_t n_words,
-             const unsigned *__restrict__ flag_bits, const unsigned *__restrict__ local,
-             const unsigned long long *__restrict__ totals, FeatureSums *out) {
-    const unsigned long long total_flags = out->nb_tot;
-    unsigned long long sum2 = 0, mn = ULLONG_MAX, mx = 0;
-    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n_rows;
-         r += (int64_t)gridDim.x * blockDim.x) {
-        unsigned long long fa = flags_before(rp[r], n_words, flag_bits, local, totals, total_flags);
-        unsigned long long fb = flags_before(rp[r + 1], n_words, flag_bits, local, totals, total_flags);
-        unsigned long long nb = fb - fa;
-        sum2 += nb * nb;
-        mn = nb < mn ? nb : mn;
-        mx = nb > mx ? nb : mx;
+    // ---- warp record for the fix-up
+    {
+        const unsigned fm = __ballot_sync(0xffffffffu, my_first_flag != kNone);
+        const long long ff = fm ? (long long)__shfl_sync(0xffffffffu, my_first_flag, __ffs(fm) - 1) : -1;
+        if (lane == 0) {
+            WarpRec rec;
+            rec.first_flag = ff;
+            rec.last_flag = c_lastflag != kNone ? (long long)c_lastflag : -1;
+            rec.nflags = c_F;
+            rec.has_rs = head_nb >= 0;
+            rec.head_nb = head_nb >= 0 ? (unsigned long long)head_nb : 0ull;
+            rec.has_open = c_Frs >= 0;                 // the last row start's row runs to the end
+            rec.open_tail = c_Frs >= 0 ? (unsigned long long)(c_F - (unsigned)c_Frs) : 0ull;
+            recs[w] = rec;
+        }
     }
-    unsigned long long sums[1] = {sum2};
-    unsigned long long *g[1] = {&out->sum_nb2};
-    block_commit<1>(sums, g, mn, &out->nb_min, mx, &out->nb_max);
+
+    // ---- commit the CTA's sums
+    __shared__ unsigned long long s_u64[6][kWarps];
+    __shared__ unsigned s_u32[7][kWarps];
+    {
+        unsigned long long v64[6] = {len2, over, nb2, sz2, (unsigned long long)n_empty, (unsigned long long)c_F};
+#pragma unroll
+        for (int i = 0; i < 5; ++i) v64[i] = warp_sum_u64(v64[i]);
+        unsigned v32[7] = {warp_min_u32(len_mn), warp_max_u32(len_mx), warp_min_u32(nb_mn), warp_max_u32(nb_mx),
+                           warp_min_u32(sz_mn), warp_max_u32(sz_mx), __reduce_or_sync(0xffffffffu, bad)};
+        if (lane == 0) {
+#pragma unroll
+            for (int i = 0; i < 6; ++i) s_u64[i][wid] = v64[i];
+#pragma unroll
+            for (int i = 0; i < 7; ++i) s_u32[i][wid] = v32[i];
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long t64[6] = {0, 0, 0, 0, 0, 0};
+        unsigned mn[3] = {UINT_MAX, UINT_MAX, UINT_MAX}, mx[3] = {0, 0, 0}, bd = 0;
+        for (int k = 0; k < kWarps; ++k) {
+            for (int i = 0; i < 6; ++i) t64[i] += s_u64[i][k];
+            for (int i = 0; i < 3; ++i) {
+                mn[i] = min(mn[i], s_u32[2 * i][k]);
+                mx[i] = max(mx[i], s_u32[2 * i + 1][k]);
+            }
+            bd |= s_u32[6][k];
+        }
+        FeatureSums &A = st->acc;
+        if (t64[0]) atomicAdd(&A.sum_len2, t64[0]);
+        if (t64[1]) atomicAdd(&A.hyb_coo_ceil, t64[1]);
+        if (t64[2]) atomicAdd(&A.sum_nb2, t64[2]);
+        if (t64[3]) atomicAdd(&A.sum_bs2, t64[3]);
+        if (t64[4]) atomicAdd(&A.n_empty, t64[4]);
+        if (t64[5]) atomicAdd(&A.nb_tot, t64[5]);
+        if (mn[0] != UINT_MAX) atomicMin(&A.len_min, (unsigned long long)mn[0]);
+        if (mx[0]) atomicMax(&A.len_max, (unsigned long long)mx[0]);
+        if (mn[1] != UINT_MAX) atomicMin(&A.nb_min, (unsigned long long)mn[1]);
+        if (mx[1]) atomicMax(&A.nb_max, (unsigned long long)mx[1]);
+        if (mn[2] != UINT_MAX) atomicMin(&A.bs_min, (unsigned long long)mn[2]);
+        if (mx[2]) atomicMax(&A.bs_max, (unsigned long long)mx[2]);
+        if (bd) atomicOr(&A.bad, (unsigned long long)bd);
+    }
+    if (use_hist) {
+        __syncthreads();
+        for (int i = threadIdx.x; i < sh_bins; i += kThreads)
+            if (s_hist[i]) atomicAdd(&hist[i], (unsigned long long)s_hist[i]);
+    }
+    // ---- the last CTA closes the open blocks/rows and writes the result
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) s_last = atomicAdd(&st->done, 1ull) == gridDim.x - 1;
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    unsigned long long fsz2 = 0, fnb2 = 0, fsz_mn = ULLONG_MAX, fsz_mx = 0, fnb_mn = ULLONG_MAX, fnb_mx = 0;
+    for (int64_t v = threadIdx.x; v < W; v += kThreads) {
+        const WarpRec rv = load_rec(recs + v);
+        if (rv.last_flag >= 0) {                 // open block: closes at the next block start
+            long long end = nnz;
+            for (int64_t u = v + 1; u < W; ++u) {
+                const long long f = __ldcg(&recs[u].first_flag);
+                if (f >= 0) { end = f; break; }
+            }
+            const unsigned long long sz = (unsigned long long)(end - rv.last_flag);
+            fsz2 += sz * sz;
+            fsz_mn = sz < fsz_mn ? sz : fsz_mn;
+            fsz_mx = sz > fsz_mx ? sz : fsz_mx;
+        }
+        if (rv.has_open) {                       // open row: closes at the next row start
+            unsigned long long nb = rv.open_tail;
+            for (int64_t u = v + 1; u < W; ++u) {
+                if (__ldcg(&recs[u].has_rs)) { nb += __ldcg(&recs[u].head_nb); break; }
+                nb += __ldcg(&recs[u].nflags);
+            }
+            fnb2 += nb * nb;
+            fnb_mn = nb < fnb_mn ? nb : fnb_mn;
+            fnb_mx = nb > fnb_mx ? nb : fnb_mx;
+        }
+    }
+    __shared__ unsigned long long s_f[6][kWarps];
+    {
+        unsigned long long a = warp_sum_u64(fsz2), b = warp_sum_u64(fnb2);
+        unsigned long long c1 = fsz_mn, c2 = fsz_mx, c3 = fnb_mn, c4 = fnb_mx;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            unsigned long long t;
+            t = __shfl_xor_sync(0xffffffffu, c1, o); c1 = t < c1 ? t : c1;
+            t = __shfl_xor_sync(0xffffffffu, c2, o); c2 = t > c2 ? t : c2;
+            t = __shfl_xor_sync(0xffffffffu, c3, o); c3 = t < c3 ? t : c3;
+            t = __shfl_xor_sync(0xffffffffu, c4, o); c4 = t > c4 ? t : c4;
+        }
+        if (lane == 0) { s_f[0][wid] = a; s_f[1][wid] = b; s_f[2][wid] = c1; s_f[3][wid] = c2; s_f[4][wid] = c3; s_f[5][wid] = c4; }
+    }
+    __syncthreads();
+    __shared__ long long s_cusp;
+    if (threadIdx.x == 0) {
+        FeatureSums R;
+        volatile FeatureSums &A = st->acc;
+        R.bad = A.bad; R.n_empty = A.n_empty; R.sum_len2 = A.sum_len2; R.len_min = A.len_min; R.len_max = A.len_max;
+        R.hyb_coo_ceil = A.hyb_coo_ceil; R.nb_tot = A.nb_tot; R.sum_nb2 = A.sum_nb2; R.nb_min = A.nb_min;
+        R.nb_max = A.nb_max; R.sum_bs2 = A.sum_bs2; R.bs_min = A.bs_min; R.bs_max = A.bs_max;
+        for (int k = 0; k < kWarps; ++k) {
+            R.sum_bs2 += s_f[0][k];
+            R.sum_nb2 += s_f[1][k];
+            R.bs_min = s_f[2][k] < R.bs_min ? s_f[2][k] : R.bs_min;
+            R.bs_max = s_f[3][k] > R.bs_max ? s_f[3][k] : R.bs_max;
+            R.nb_min = s_f[4][k] < R.nb_min ? s_f[4][k] : R.nb_min;
+            R.nb_max = s_f[5][k] > R.nb_max ? s_f[5][k] : R.nb_max;
+        }
+        if (R.n_empty > 0) R.nb_min = 0;        // an empty row has no block (A8: all rows)
+        st->result = R;
+        s_cusp = (long long)R.len_max;
+    }
+    __syncthreads();
+    if (use_hist) {
+        // A2 "cusp" width: smallest k < nnz_max with 3*#{len>k} < n or #{len>k} < 4096, else
+        // nnz_max; #{len>k} = n - sum_{j<=k} hist[j], exact for k < hist_bins - 1 and the
+        // answer is < hist_bins - 1 by construction (hist_bins = nnz/4096 + 2).
+        const long long kmax = s_cusp;
+        const unsigned long long empty_rows = st->result.n_empty;
+        __shared__ unsigned long long s_scan[kWarps];
+        __shared__ unsigned long long s_run;
+        __shared__ long long s_ans;
+        if (threadIdx.x == 0) { s_run = 0; s_ans = kmax; }
+        __syncthreads();
+        for (long long b0 = 0; b0 < kmax && b0 < hist_bins; b0 += kThreads) {
+            const long long k = b0 + threadIdx.x;
+            const unsigned long long hv = k == 0 ? (unsigned long long)empty_rows : (k < hist_bins ? __ldcg(hist + k) : 0ull);
+            unsigned long long incl = hv;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const unsigned long long t = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += t;
+            }
+            if (lane == 31) s_scan[wid] = incl;
+            __syncthreads();
+            unsigned long long woff = 0;
+            for (int j = 0; j < wid; ++j) woff += s_scan[j];
+            const unsigned long long cum = s_run + woff + incl;     // sum_{j<=k} hist[j]
+            const long long longer = n - (long long)cum;
+            const bool hit = k < kmax && k < hist_bins && (3 * longer < n || longer < 4096);
+            const unsigned hb = __ballot_sync(0xffffffffu, hit);
+            if (hb && lane == __ffs(hb) - 1) atomicMin((unsigned long long *)&s_ans, (unsigned long long)k);
+            __syncthreads();
+            if (threadIdx.x == kThreads - 1) s_run += woff + incl;
+            __syncthreads();
+            if (s_ans < kmax) break;
+        }
+        if (threadIdx.x == 0) st->cusp = n > 0 ? s_ans : 0;
+        for (long long k = threadIdx.x; k < hist_bins; k += kThreads) hist[k] = 0ull;
+    }
+    if (threadIdx.x == 0) {
+        init_sums(st->acc);
+        st->done = 0;
+    }
 }
 
-int grid_for(const spmv_ctx *ctx, int64_t work, int per_block = kThreads) {
-    int64_t g = ceil_div<int64_t>(work, per_block);
-    int64_t cap = (int64_t)ctx->sm_count * 8;
-    if (g > cap) g = cap;
-    if (g < 1) g = 1;
-    return (int)g;
+__global__ void k_features_state_init(FeatureState *st) {
+    init_sums(st->acc);
+    st->done = 0;
+    st->cusp = 0;
 }
 
 template <typename IT>
@@ -368,75 +709,50 @@ spmv_status feature_pass_t(spmv_ctx *ctx, const spmv_csr *A, cudaStream_t s, int
                            FeatureSums *host, int64_t *hyb_cusp) {
     const IT *rp = reinterpret_cast<const IT *>(A->row_ptr);
     const int64_t n = A->n_rows, nnz = A->nnz;
-    const int64_t n_words = ceil_div<int64_t>(nnz, 32);
-    const int64_t n_chunks = ceil_div<int64_t>(n_words, kScanChunk);
-    const int64_t kh = n > 0 ? ceil_div<int64_t>(nnz, n) : 0;
+    const int64_t items = (int64_t)kRowW * n + nnz;
     const int64_t hist_bins = level ? nnz / 4096 + 2 : 0;
+    std::lock_guard<std::mutex> lock(ctx->feat_mu);
 
-    Scratch sums(ctx, s), rs(ctx, s), flags(ctx, s), local(ctx, s), totals(ctx, s), hist(ctx, s);
-    SPMV_TRY(sums.alloc(sizeof(FeatureSums)));
-    SPMV_TRY(rs.alloc(n_words * 4));
-    const int64_t n_words_pad = ceil_div<int64_t>(n_words, 256) * 256 + 256;   // F4 reads whole 256-word chunks
-    SPMV_TRY(flags.alloc(n_words_pad * 4));
-    if (level) {
-        SPMV_TRY(local.alloc(n_words * 4));
-        SPMV_TRY(totals.alloc(n_chunks * 8));
-        SPMV_TRY(hist.alloc(hist_bins * 8));
-        SPMV_CUDA_TRY(cudaMemsetAsync(hist.p, 0, hist_bins * 8, s));
-    }
-    FeatureSums init{};
-    init.len_min = init.nb_min = init.bs_min = ULLONG_MAX;
-    SPMV_CUDA_TRY(cudaMemcpyAsync(sums.p, &init, sizeof(init), cudaMemcpyHostToDevice, s));
-    SPMV_CUDA_TRY(cudaMemsetAsync(rs.p, 0, n_words * 4, s));
-    SPMV_CUDA_TRY(cudaMemsetAsync(flags.p, 0, n_words_pad * 4, s));
-    FeatureSums *d = sums.as<FeatureSums>();
-
-    if (n >= 0) {
-        k_rows<IT><<<grid_for(ctx, n > 0 ? n : 1), kThreads, 0, s>>>(
-            rp, n, nnz, kh, rs.as<unsigned>(), level ? hist.as<unsigned long long>() : nullptr,
-            hist_bins, d);
+    // ctx-owned state, allocated once (and the histogram grown on demand)
+    const int64_t max_ctas = (int64_t)ctx->sm_count * kCtasPerSm;
+    if (!ctx->feat_state) {
+        SPMV_TRY(dev_alloc(ctx, sizeof(FeatureState), nullptr, &ctx->feat_state));
+        SPMV_TRY(dev_alloc(ctx, max_ctas * kWarps * sizeof(WarpRec), nullptr, &ctx->feat_recs));
+        SPMV_CUDA_TRY(cudaMallocHost(&ctx->feat_host, sizeof(FeatureState)));
+        k_features_state_init<<<1, 1, 0, nullptr>>>(reinterpret_cast<FeatureState *>(ctx->feat_state));
         SPMV_LAUNCH_CHECK();
+        SPMV_CUDA_TRY(cudaStreamSynchronize(nullptr));
     }
-    if (n_words > 0) {
-        k_flags<<<grid_for(ctx, ceil_div<int64_t>(n_words, kChunkWords) * 32), kThreads, 0, s>>>(A->col_idx, nnz, A->n_cols, n_words,
-                                                                rs.as<unsigned>(), flags.as<unsigned>(), d);
-        SPMV_LAUNCH_CHECK();
+    if (hist_bins * 8 > (int64_t)ctx->feat_hist_bytes) {
+        if (ctx->feat_hist) dev_free(ctx, ctx->feat_hist, ctx->feat_hist_bytes, nullptr);
+        ctx->feat_hist = nullptr;
+        ctx->feat_hist_bytes = 0;
+        SPMV_TRY(dev_alloc(ctx, hist_bins * 8, nullptr, &ctx->feat_hist));
+        ctx->feat_hist_bytes = hist_bins * 8;
+        SPMV_CUDA_TRY(cudaMemsetAsync(ctx->feat_hist, 0, hist_bins * 8, nullptr));
+        SPMV_CUDA_TRY(cudaStreamSynchronize(nullptr));
     }
-    if (level && n_words > 0) {
-        k_scan_local<<<(unsigned)n_chunks, kThreads, 0, s>>>(flags.as<unsigned>(), n_words, local.as<unsigned>(),
-                                                             totals.as<unsigned long long>());
-        SPMV_LAUNCH_CHECK();
-        k_scan_totals<<<1, kThreads, 0, s>>>(totals.as<unsigned long long>(), n_chunks);
-        SPMV_LAUNCH_CHECK();
-        k_block_sizes<<<grid_for(ctx, ceil_div<int64_t>(n_words, 32 * kLaneWords) * 32), kThreads, 0, s>>>(flags.as<unsigned>(), n_words, nnz, d);
-        SPMV_LAUNCH_CHECK();
-    }
-    if (level && n > 0) {
-        k_row_blocks<IT><<<grid_for(ctx, n), kThreads, 0, s>>>(rp, n, n_words, flags.as<unsigned>(),
-                                                               local.as<unsigned>(),
-                                                               totals.as<unsigned long long>(), d);
-        SPMV_LAUNCH_CHECK();
-    }
-    SPMV_CUDA_TRY(cudaMemcpyAsync(host, d, sizeof(FeatureSums), cudaMemcpyDeviceToHost, s));
-    std::vector<unsigned long long> h;
-    if (level) {
-        h.resize(hist_bins);
-        SPMV_CUDA_TRY(cudaMemcpyAsync(h.data(), hist.p, hist_bins * 8, cudaMemcpyDeviceToHost, s));
-    }
+    // grid: up to kCtasPerSm resident CTAs per SM, each warp >= one sub-span of work
+    int64_t ctas = ceil_div<int64_t>(items > 0 ? items : 1, (int64_t)kWarps * kSub);
+    if (ctas > max_ctas) ctas = max_ctas;
+    if (ctas < 1) ctas = 1;
+    const int64_t W = ctas * kWarps;
+    const int64_t per_warp = ceil_div<int64_t>(items > 0 ? items : 1, W);
+    FeatureState *st = reinterpret_cast<FeatureState *>(ctx->feat_state);
+    k_features<IT><<<(unsigned)ctas, kThreads, 0, s>>>(
+        rp, A->col_idx, n, nnz, A->n_cols, n > 0 ? ceil_div<int64_t>(nnz, n) : 0, per_warp,
+        reinterpret_cast<WarpRec *>(ctx->feat_recs), level ? reinterpret_cast<unsigned long long *>(ctx->feat_hist) : nullptr,
+        hist_bins, st);
+    SPMV_LAUNCH_CHECK();
+    FeatureState *hs = reinterpret_cast<FeatureState *>(ctx->feat_host);
+    SPMV_CUDA_TRY(cudaMemcpyAsync(&hs->result, &st->result, sizeof(FeatureSums) + sizeof(long long),
+                                  cudaMemcpyDeviceToHost, s));
     SPMV_CUDA_TRY(cudaStreamSynchronize(s));
+    *host = hs->result;
     if (n == 0) { host->len_min = 0; host->len_max = 0; }
     if (nnz == 0) { host->nb_tot = 0; host->sum_bs2 = 0; host->bs_min = 0; host->bs_max = 0; }
-    if (level && n > 0 && nnz == 0) { host->nb_min = 0; host->nb_max = 0; host->sum_nb2 = 0; }
-    if (hyb_cusp) {
-        // A2 "cusp" width: smallest k with 3*#{len>k} < n_rows or #{len>k} < 4096,
-        // else the maximum row length; #{len>k} is exact for k <= nnz/4096.
-        int64_t kmax = (int64_t)host->len_max, longer = n, ans = kmax;
-        for (int64_t k = 0; level && k < kmax; ++k) {
-            longer -= (int64_t)h[k < hist_bins - 1 ? k : hist_bins - 1];
-            if (3 * longer < n || longer < 4096) { ans = k; break; }
-        }
-        *hyb_cusp = n > 0 ? ans : 0;
-    }
+    if (n > 0 && nnz == 0) { host->nb_min = 0; host->nb_max = 0; host->sum_nb2 = 0; }
+    if (hyb_cusp) *hyb_cusp = level ? hs->cusp : 0;
     return SPMV_OK;
 }
 
@@ -446,6 +762,15 @@ spmv_status feature_pass(spmv_ctx *ctx, const spmv_csr *A, cudaStream_t s, int l
                          int64_t *hyb_cusp) {
     if (A->ptr_type == SPMV_I32) return feature_pass_t<int>(ctx, A, s, level, out, hyb_cusp);
     return feature_pass_t<int64_t>(ctx, A, s, level, out, hyb_cusp);
+}
+
+void feature_state_free(spmv_ctx *ctx) {
+    if (ctx->feat_state) dev_free(ctx, ctx->feat_state, sizeof(FeatureState), nullptr);
+    if (ctx->feat_recs) dev_free(ctx, ctx->feat_recs, (size_t)ctx->sm_count * kCtasPerSm * kWarps * sizeof(WarpRec), nullptr);
+    if (ctx->feat_hist) dev_free(ctx, ctx->feat_hist, ctx->feat_hist_bytes, nullptr);
+    if (ctx->feat_host) cudaFreeHost(ctx->feat_host);
+    ctx->feat_state = ctx->feat_recs = ctx->feat_hist = ctx->feat_host = nullptr;
+    ctx->feat_hist_bytes = 0;
 }
 
 // A9: fixed fp64 formulas from exact integer sums (identical rounding on every run).

@@ -1,5 +1,6 @@
 // internal.h -- ctx/handle layout and the internal entry points of libspmv.
 #pragma once
+#include <mutex>
 #include "common.cuh"
 
 struct spmv_ctx {
@@ -8,6 +9,12 @@ struct spmv_ctx {
     int64_t l2_bytes = 0;
     spmv_allocator alloc{};
     bool has_alloc = false;
+    // feature pass state (features.cu): device accumulators + per-warp records + the A2
+    // histogram, allocated once and reset by the kernel itself; pinned result readback.
+    // The pass blocks until done; the mutex serialises callers sharing the ctx.
+    std::mutex feat_mu;
+    void *feat_state = nullptr, *feat_recs = nullptr, *feat_hist = nullptr, *feat_host = nullptr;
+    size_t feat_hist_bytes = 0;
 };
 
 namespace spmv {
@@ -57,6 +64,7 @@ spmv_status feature_pass(spmv_ctx *ctx, const spmv_csr *A, cudaStream_t s, int l
                          FeatureSums *out, int64_t *hyb_cusp);
 void finalize_features(const spmv_csr *A, const FeatureSums &fs, int64_t hyb_cusp,
                        spmv_features_t *f);
+void feature_state_free(spmv_ctx *ctx);
 
 }  // namespace spmv
 

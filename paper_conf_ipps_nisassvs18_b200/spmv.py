@@ -73,7 +73,8 @@ PAPER_FEATURES = ("n_rows", "n_cols", "nnz_tot", "nnz_mu", "nnz_frac",          
 class spmv_convert_opts(C.Structure):
     _fields_ = [("hyb_rule", C.c_int), ("hyb_width", C.c_int64), ("csr5_sigma", C.c_int),
                 ("merge_items", C.c_int), ("vector_width", C.c_int), ("max_bytes", C.c_size_t),
-                ("alias_input", C.c_int), ("index64", C.c_int), ("csr_chunk", C.c_int64)]
+                ("alias_input", C.c_int), ("index64", C.c_int), ("csr_chunk", C.c_int64),
+                ("features", C.POINTER(spmv_features_t))]
 
 
 class spmv_handle_info(C.Structure):
@@ -263,6 +264,12 @@ def convert_opts(**kw) -> spmv_convert_opts:
     for k, v in kw.items():
         if k == "hyb_rule" and isinstance(v, str):
             v = rules[v]
+        if k == "features":
+            if v is None:
+                continue
+            ft = spmv_features_t(**{name: v[name] for name, _ in spmv_features_t._fields_})
+            o._features_keep = ft                      # alive as long as the opts struct
+            v = C.pointer(ft)
         setattr(o, k, v)
     return o
 

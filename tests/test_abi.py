@@ -33,7 +33,7 @@ def test_every_declared_symbol_is_exported(L):
 
 
 def test_abi_version_and_status_strings(L):
-    assert L.spmv_abi_version() == 2
+    assert L.spmv_abi_version() == 3
     for code, name in [(0, b"SPMV_OK"), (2, b"SPMV_ERR_NOT_CANONICAL"), (3, b"SPMV_ERR_SIZE"),
                        (6, b"SPMV_ERR_UNSUPPORTED")]:
         assert L.spmv_status_str(code) == name
