@@ -298,6 +298,19 @@ spmv_status spmv_slice_split(spmv_ctx *ctx, const spmv_csr *A, const int64_t *ro
                              int part, const int32_t *colmap, int which, void *stream, int32_t *row_ptr_out,
                              int32_t *col_out, void *vals_out, int64_t *nnz_out);
 
+/* Halo exchange of a row partition: the receiver `part`
+ * needs, from every other owner o, exactly the x entries of o's rows (= columns, square A)
+ * that part's rows reference.  colmap_out[j] (DEVICE int32[n_cols]) = owner(j)*S +
+ * (number of such columns of owner(j) below j) for every column j referenced by a row of
+ * `part` and owned by another part, -1 otherwise, with S = max(1, max_o counts[o]) the
+ * receiver's slot (host output *slot); counts_host[nparts] (HOST) receives the per-owner
+ * counts (counts_host[part] = 0).  The receive buffer of `part` holds owner o's entries at
+ * [o*S, o*S + counts[o]).  The sender's pack list for this receiver is
+ * spmv_colmap_pack_index(colmap_out, ..., sender, S).  Identical on every rank.  Blocks on
+ * `stream` (one readback). */
+spmv_status spmv_halo_colmap(spmv_ctx *ctx, const spmv_csr *A, const int64_t *row_splits_host, int nparts,
+                             int part, void *stream, int32_t *colmap_out, int64_t *counts_host, int64_t *slot);
+
 /* dst[q] = src[idx[q]] for q < n (DEVICE arrays of `dtype`): the per-step packing of a
  * rank's x slice into its compressed slot.  Asynchronous. */
 spmv_status spmv_gather(spmv_ctx *ctx, spmv_dtype dtype, const void *src, const int32_t *idx, int64_t n,

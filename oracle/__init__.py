@@ -91,6 +91,7 @@ def lib():
             "ora_partition_slot": (_i64, [_p, C.c_int]),
             "ora_slice_remap": (C.c_int, [_i64, _p, _p, _p, _p, C.c_int, C.c_int, _p, _p, _p]),
             "ora_partition_colmap": (_i64, [_i64, _p, _p, _p, C.c_int, _p]),
+            "ora_halo_colmap": (_i64, [_i64, _p, _p, _p, C.c_int, C.c_int, _p, _p]),
             "ora_slice_remap_colmap": (C.c_int, [_i64, _p, _p, _p, _p, C.c_int, _p, _p, _p, _p]),
             "ora_slice_split": (_i64, [_i64, _p, _p, _p, _p, C.c_int, C.c_int, _p, C.c_int, _p, _p, _p]),
         }
@@ -334,6 +335,26 @@ def partition_colmap(A, splits):
     S = lib().ora_partition_colmap(A.n_rows, _ptr(A.row_ptr), _ptr(A.col), _ptr(s), s.size - 1, _ptr(cm))
     assert S >= 0
     return cm, int(S)
+
+
+def halo_colmap(A, splits, part):
+    """Halo map of receiver `part`: (colmap int32[n], counts int64[P], S)."""
+    A = CSR.of(A)
+    s = _c(splits, np.int64)
+    cm = _buf(A.n_rows, np.int32)
+    cnt = _buf(s.size - 1, np.int64)
+    S = lib().ora_halo_colmap(A.n_rows, _ptr(A.row_ptr), _ptr(A.col), _ptr(s), s.size - 1, int(part), _ptr(cm),
+                              _ptr(cnt))
+    assert S >= 1
+    return cm, cnt, int(S)
+
+
+def halo_pack_index(colmap, splits, sender, S):
+    """Sender's pack list for the receiver of `colmap`: local indices j - splits[sender] of
+    the sender's columns the receiver references, in slot order (plain loop)."""
+    s = np.asarray(splits, np.int64)
+    out = [j - int(s[sender]) for j in range(int(s[sender]), int(s[sender + 1])) if colmap[j] >= 0]
+    return np.asarray(out, dtype=np.int32)
 
 
 def slice_remap_colmap(A, splits, part, colmap):

@@ -602,6 +602,36 @@ int64_t ora_partition_colmap(int64_t n_rows, const int64_t *row_ptr, const int32
     return S;
 }
 
+/* Halo exchange: receiver `part` needs the columns its rows reference
+ * that other parts own.  Plain loops: mark them, count per owner, S = max(1, max count),
+ * colmap[j] = owner*S + (rank of j among the owner's marked columns), -1 elsewhere.
+ * counts[o] = marked columns of owner o.  Returns S. */
+int64_t ora_halo_colmap(int64_t n_rows, const int64_t *row_ptr, const int32_t *col, const int64_t *splits,
+                        int nparts, int part, int32_t *colmap, int64_t *counts)
+{
+    unsigned char *used = (unsigned char *)calloc((size_t)(n_rows > 0 ? n_rows : 1), 1);
+    if (!used) return -1;
+    for (int64_t r = splits[part]; r < splits[part + 1]; ++r)
+        for (int64_t k = row_ptr[r]; k < row_ptr[r + 1]; ++k) {
+            int64_t j = col[k];
+            if (j < splits[part] || j >= splits[part + 1]) used[j] = 1;
+        }
+    int64_t S = 1;
+    for (int o = 0; o < nparts; ++o) {
+        int64_t c = 0;
+        for (int64_t j = splits[o]; j < splits[o + 1]; ++j) c += used[j];
+        counts[o] = c;
+        if (c > S) S = c;
+    }
+    for (int o = 0; o < nparts; ++o) {
+        int64_t c = 0;
+        for (int64_t j = splits[o]; j < splits[o + 1]; ++j)
+            colmap[j] = used[j] ? (int32_t)(o * S + c++) : -1;
+    }
+    free(used);
+    return S;
+}
+
 int ora_slice_remap_colmap(int64_t n_rows, const int64_t *row_ptr, const int32_t *col,
                            const double *val, const int64_t *splits, int part, const int32_t *colmap,
                            int64_t *out_row_ptr, int32_t *out_col, double *out_val)

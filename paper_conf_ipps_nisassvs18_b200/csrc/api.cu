@@ -391,6 +391,18 @@ spmv_status spmv_slice_remap_colmap(spmv_ctx *ctx, const spmv_csr *A, const int6
     return slice_remap_colmap_impl(ctx, A, splits, nparts, part, colmap, as_stream(stream), rp_out, col_out, val_out);
 }
 
+spmv_status spmv_halo_colmap(spmv_ctx *ctx, const spmv_csr *A, const int64_t *splits, int nparts, int part,
+                             void *stream, int32_t *colmap_out, int64_t *counts_host, int64_t *slot) {
+    if (!ctx || !splits || nparts <= 0 || part < 0 || part >= nparts || !colmap_out || !counts_host || !slot) {
+        set_error("bad args");
+        return SPMV_ERR_INVALID_ARG;
+    }
+    SPMV_TRY(check_csr(A));
+    if (A->n_rows != A->n_cols) { set_error("halo_colmap needs a square matrix"); return SPMV_ERR_INVALID_ARG; }
+    SPMV_ON_DEVICE(ctx->device);
+    return halo_colmap_impl(ctx, A, splits, nparts, part, as_stream(stream), colmap_out, counts_host, slot);
+}
+
 spmv_status spmv_colmap_pack_index(spmv_ctx *ctx, const int32_t *colmap, const int64_t *splits, int nparts, int part,
                                    int64_t slot, void *stream, int32_t *idx_out, int64_t *count) {
     if (!ctx || !colmap || !splits || nparts <= 0 || part < 0 || part >= nparts || !count || slot < 0) {

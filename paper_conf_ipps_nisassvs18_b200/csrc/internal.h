@@ -114,6 +114,8 @@ spmv_status colmap_impl(spmv_ctx *ctx, const spmv_csr *A, const int64_t *splits,
 spmv_status slice_remap_colmap_impl(spmv_ctx *ctx, const spmv_csr *A, const int64_t *splits, int nparts, int part,
                                     const int32_t *colmap, cudaStream_t s, int32_t *rp_out, int32_t *col_out,
                                     void *val_out);
+spmv_status halo_colmap_impl(spmv_ctx *ctx, const spmv_csr *A, const int64_t *splits, int nparts, int part,
+                             cudaStream_t s, int32_t *colmap, int64_t *counts, int64_t *slot);
 spmv_status pack_index_impl(spmv_ctx *ctx, const int32_t *colmap, const int64_t *splits, int nparts, int part,
                             int64_t slot, cudaStream_t s, int32_t *idx, int64_t *count);
 spmv_status gather_impl(spmv_ctx *ctx, spmv_dtype dt, const void *src, const int32_t *idx, int64_t n, void *dst,

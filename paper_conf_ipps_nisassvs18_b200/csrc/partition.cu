@@ -72,6 +72,13 @@ __global__ void k_mark_used(const int *col, int64_t nnz, unsigned char *used) {
     for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nnz; k += (int64_t)gridDim.x * blockDim.x)
         used[__ldg(col + k)] = 1;                 // benign race: every writer stores 1
 }
+// halo: columns referenced by the rows [rp[r0], rp[r1]) of one part, outside its own range
+__global__ void k_mark_foreign(const int *col, int64_t k0, int64_t k1, int64_t c0, int64_t c1, unsigned char *used) {
+    for (int64_t k = k0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < k1; k += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t j = __ldg(col + k);
+        if (j < c0 || j >= c1) used[j] = 1;       // benign race: every writer stores 1
+    }
+}
 __global__ void k_used_to_i64(const unsigned char *used, int64_t n, int64_t *out) {
     for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
         out[j] = used[j];
@@ -186,6 +193,50 @@ spmv_status colmap_impl(spmv_ctx *ctx, const spmv_csr *A, const int64_t *sp, int
     int64_t S = 0;
     for (int k = 0; k < nparts; ++k) S = std::max(S, at[k + 1] - at[k]);
     if ((int64_t)nparts * S > (int64_t)INT32_MAX) { set_error("compressed slots exceed int32"); return SPMV_ERR_SIZE; }
+    Splits spl{};
+    for (int k = 0; k <= nparts; ++k) spl.s[k] = sp[k];
+    spl.nparts = nparts;
+    spl.slot = S;
+    if (n) {
+        k_colmap<<<blocks_for(ctx, n), 256, 0, s>>>(used.as<unsigned char>(), prefix.as<int64_t>(), n, spl, colmap);
+        SPMV_LAUNCH_CHECK();
+    }
+    *slot = S;
+    return SPMV_OK;
+}
+
+spmv_status halo_colmap_impl(spmv_ctx *ctx, const spmv_csr *A, const int64_t *sp, int nparts, int part,
+                             cudaStream_t s, int32_t *colmap, int64_t *counts, int64_t *slot) {
+    SPMV_TRY(check_splits(A, sp, nparts));
+    const int64_t n = A->n_cols;
+    Scratch used(ctx, s), u64(ctx, s), prefix(ctx, s);
+    SPMV_TRY(used.alloc(std::max<int64_t>(n, 1)));
+    SPMV_TRY(u64.alloc(std::max<int64_t>(n, 1) * 8));
+    SPMV_TRY(prefix.alloc((n + 1) * 8));
+    SPMV_CUDA_TRY(cudaMemsetAsync(used.p, 0, std::max<int64_t>(n, 1), s));
+    int64_t k0 = 0, k1 = 0;
+    SPMV_TRY(rp_at(A, sp[part], s, &k0));
+    SPMV_TRY(rp_at(A, sp[part + 1], s, &k1));
+    if (k1 > k0) {
+        k_mark_foreign<<<blocks_for(ctx, k1 - k0), 256, 0, s>>>(A->col_idx, k0, k1, sp[part], sp[part + 1],
+                                                               used.as<unsigned char>());
+        SPMV_LAUNCH_CHECK();
+    }
+    if (n) {
+        k_used_to_i64<<<blocks_for(ctx, n), 256, 0, s>>>(used.as<unsigned char>(), n, u64.as<int64_t>());
+        SPMV_LAUNCH_CHECK();
+    }
+    SPMV_TRY(exclusive_scan_i64(ctx, u64.as<int64_t>(), prefix.as<int64_t>(), n, s));
+    std::vector<int64_t> at(nparts + 1);
+    for (int k = 0; k <= nparts; ++k)
+        SPMV_CUDA_TRY(cudaMemcpyAsync(&at[k], prefix.as<int64_t>() + sp[k], 8, cudaMemcpyDeviceToHost, s));
+    SPMV_CUDA_TRY(cudaStreamSynchronize(s));
+    int64_t S = 1;
+    for (int k = 0; k < nparts; ++k) {
+        counts[k] = at[k + 1] - at[k];
+        S = std::max(S, counts[k]);
+    }
+    if ((int64_t)nparts * S > (int64_t)INT32_MAX) { set_error("halo slots exceed int32"); return SPMV_ERR_SIZE; }
     Splits spl{};
     for (int k = 0; k <= nparts; ++k) spl.s[k] = sp[k];
     spl.nparts = nparts;

@@ -135,6 +135,8 @@ def lib():
             "spmv_colmap_pack_index": (C.c_int, [_P, _P, C.POINTER(C.c_int64), C.c_int, C.c_int, C.c_int64, _P, _P,
                                                  C.POINTER(C.c_int64)]),
             "spmv_gather": (C.c_int, [_P, C.c_int, _P, _P, C.c_int64, _P, _P]),
+            "spmv_halo_colmap": (C.c_int, [_P, C.POINTER(spmv_csr), C.POINTER(C.c_int64), C.c_int, C.c_int, _P, _P,
+                                           C.POINTER(C.c_int64), C.POINTER(C.c_int64)]),
             "spmv_slice_split": (C.c_int, [_P, C.POINTER(spmv_csr), C.POINTER(C.c_int64), C.c_int, C.c_int, _P,
                                            C.c_int, _P, _P, _P, _P, C.POINTER(C.c_int64)]),
             "spmv_status_str": (C.c_char_p, [C.c_int]),
@@ -370,6 +372,21 @@ def spmv_colmap_pack_index(colmap: torch.Tensor, splits, part: int, slot: int, s
     _check(lib().spmv_colmap_pack_index(ctx.ptr, colmap.data_ptr(), csp, sp.size - 1, int(part), int(slot),
                                         _stream_ptr(stream), idx.data_ptr(), C.byref(cnt)))
     return idx[: cnt.value]
+
+
+def spmv_halo_colmap(A: CSR, splits, part: int, stream=None):
+    """Halo map of receiver `part`: (int32 device colmap[n_cols], per-owner
+    counts (numpy int64), slot S)."""
+    ctx = context(A.row_ptr.device.index)
+    sp, csp = _splits_c(splits)
+    P = sp.size - 1
+    colmap = torch.empty(max(A.n_cols, 1), dtype=torch.int32, device=A.row_ptr.device)
+    counts = np.zeros(P, dtype=np.int64)
+    slot = C.c_int64()
+    a = A.as_c()
+    _check(lib().spmv_halo_colmap(ctx.ptr, C.byref(a), csp, P, int(part), _stream_ptr(stream), colmap.data_ptr(),
+                                  counts.ctypes.data_as(C.POINTER(C.c_int64)), C.byref(slot)))
+    return colmap[: A.n_cols], counts, slot.value
 
 
 def spmv_slice_split(A: CSR, splits, part: int, which: int, colmap: Optional[torch.Tensor] = None,

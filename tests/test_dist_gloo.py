@@ -109,6 +109,19 @@ def test_layout_host_logic():
     assert lay0.pack_x(torch.ones(3, dtype=torch.float64)).tolist() == [1, 1, 1, 0, 0, 0, 0]
 
 
+class OracleHaloIndex:
+    """The halo plan's index maps from the oracle (CPU test stand-in for libspmv's
+    spmv_halo_colmap / spmv_colmap_pack_index, which are pinned to it on the GPU)."""
+
+    @staticmethod
+    def colmap(A, splits, k):
+        return oracle.halo_colmap(A, splits, k)
+
+    @staticmethod
+    def pack(colmap, splits, rank, S):
+        return oracle.halo_pack_index(colmap, splits, rank, S)
+
+
 def _halo_worker(rank, world, port, case, q):
     """HaloPlan over gloo: pack, all_to_all_single, own + foreign blocks
     (oracle SpMV per block), integer regime so the split sum is exact."""
@@ -127,7 +140,7 @@ def _halo_worker(rank, world, port, case, q):
         y = matgen.vector(A.n_rows, 9, 2, "int")
         splits = oracle.partition(A, world)
         lay = ShardLayout(splits, rank)
-        plan = HaloPlan(torch.from_numpy(A.row_ptr), torch.from_numpy(A.col.astype(np.int64)), A.n_cols, splits, rank)
+        plan = HaloPlan(A, splits, rank, index=OracleHaloIndex)
         x_own = torch.from_numpy(x[lay.r0:lay.r1].copy())
         send = x_own[plan.send_index.to(torch.int64)].contiguous()          # spmv_gather's job on the GPU
         recv = torch.zeros(plan.recv_len, dtype=torch.float64)
@@ -137,7 +150,7 @@ def _halo_worker(rank, world, port, case, q):
         cols, vals = A.col[a:b], A.val[a:b]
         rows = np.repeat(np.arange(lay.rows), np.diff(A.row_ptr[lay.r0:lay.r1 + 1]))
         mine = (cols >= lay.r0) & (cols < lay.r1)
-        cm = plan.colmap.numpy()
+        cm = np.asarray(plan.colmap)
         assert np.all(cm[cols[~mine]] >= 0)
 
         def block(sel, c, ncols):

@@ -203,7 +203,7 @@ def test_halo_virtual(sp, case, fmt, P):
     dA = sp.CSR.from_host(A)
     splits = sp.partition(dA, P)
     lays = [ShardLayout(splits, k) for k in range(P)]
-    plans = [HaloPlan(dA.row_ptr, dA.col, A.n_cols, splits, k) for k in range(P)]
+    plans = [HaloPlan(dA, splits, k) for k in range(P)]
     xd = torch.from_numpy(x).cuda()
     sends = []
     for k, lay in enumerate(lays):
@@ -254,3 +254,29 @@ def test_halospmv_nccl_world1(sp):
         assert ok, (nbad, ratio)
     finally:
         dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 5, 8])
+@pytest.mark.parametrize("case", ["lap96", "rmat12", "empty_runs"])
+def test_halo_colmap_bit_exact(sp, case, P):
+    """spmv_halo_colmap + spmv_colmap_pack_index (the halo plan's index maps) bit-exact
+    against the oracle's plain loops, for every receiver and sender."""
+    from paper_conf_ipps_nisassvs18_b200.spmv import spmv_colmap_pack_index, spmv_halo_colmap
+    if case == "lap96":
+        A = matgen.laplacian5(96)
+    elif case == "rmat12":
+        A = matgen.rmat(12, seed=46)
+    else:
+        lens = np.random.default_rng(46).integers(0, 9, 4000)
+        lens[100:900] = 0
+        A = matgen.from_lengths(lens, 4000, seed=46)
+    dA = sp.CSR.from_host(A)
+    splits = sp.partition(dA, P)
+    for k in range(P):
+        cm, counts, S = spmv_halo_colmap(dA, splits, k)
+        cmo, cnto, So = oracle.halo_colmap(A, splits, k)
+        assert S == So and np.array_equal(counts, cnto)
+        assert np.array_equal(cm.cpu().numpy(), cmo)
+        for snd in range(P):
+            idx = spmv_colmap_pack_index(cm, splits, snd, S).cpu().numpy()
+            assert np.array_equal(idx, oracle.halo_pack_index(cmo, splits, snd, So)), (k, snd)

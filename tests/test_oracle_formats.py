@@ -494,3 +494,51 @@ def test_csr_chunks_tile_long_rows(C):
             assert lo.tolist() == list(range(a, b, C))
             parts = [np.sum(A.val[k:min(k + C, b)] * x[A.col[k:min(k + C, b)]]) for k in lo]
             assert abs(sum(parts) - np.sum(A.val[a:b] * x[A.col[a:b]])) <= 1e-12 * np.sum(np.abs(A.val[a:b] * x[A.col[a:b]])) + 1e-300
+
+
+def _halo_brute(A, splits, k):
+    """Receiver k's halo by sets: foreign columns referenced by k's rows, per owner sorted."""
+    s = np.asarray(splits, np.int64)
+    P = s.size - 1
+    a, b = int(A.row_ptr[s[k]]), int(A.row_ptr[s[k + 1]])
+    cols = np.unique(A.col[a:b].astype(np.int64))
+    owner = np.searchsorted(s, cols, side="right") - 1
+    cols, owner = cols[owner != k], owner[owner != k]
+    counts = np.bincount(owner, minlength=P).astype(np.int64)
+    S = max(1, int(counts.max()) if counts.size else 1)
+    cm = np.full(A.n_cols, -1, np.int32)
+    for o in range(P):
+        mine = cols[owner == o]
+        cm[mine] = o * S + np.arange(mine.size)
+    return cm, counts, S
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 7])
+@pytest.mark.parametrize("case", ["lap30", "rmat10", "band", "ragged"])
+def test_oracle_halo_colmap_brute_force(case, P):
+    """ora_halo_colmap == a set-based brute force; every referenced
+    foreign column lands in its owner's slot range, distinct and in column order."""
+    if case == "lap30":
+        A = matgen.laplacian5(30)
+    elif case == "rmat10":
+        A = matgen.rmat(10, seed=3)
+    elif case == "band":
+        A = matgen.window(700, 700, 6, 0.7, seed=5, mode=0)
+    else:
+        lens = np.random.default_rng(8).integers(0, 9, 900)
+        lens[50:300] = 0
+        lens[600] = 800
+        A = matgen.from_lengths(lens, 900, seed=8)
+    splits = oracle.partition(A, P)
+    for k in range(P):
+        cm, cnt, S = oracle.halo_colmap(A, splits, k)
+        cmb, cntb, Sb = _halo_brute(A, splits, k)
+        assert S == Sb and np.array_equal(cnt, cntb) and np.array_equal(cm, cmb), (case, P, k)
+        for snd in range(P):
+            idx = oracle.halo_pack_index(cm, splits, snd, S)
+            assert idx.size == cnt[snd]
+            js = idx.astype(np.int64) + int(splits[snd])
+            assert np.all(np.diff(js) > 0)
+            assert np.array_equal(cm[js], snd * S + np.arange(idx.size))
+    if case == "lap30" and P > 1:
+        assert max(oracle.halo_colmap(A, splits, k)[2] for k in range(P)) <= 30   # one grid line

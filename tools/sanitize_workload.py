@@ -83,7 +83,7 @@ def main():
             S.spmv_slice_split(dA, splits, part, which)
         # halo exchange plumbing: the foreign block through a HaloPlan colmap
         from paper_conf_ipps_nisassvs18_b200.dist import HaloPlan
-        plan = HaloPlan(dA.row_ptr, dA.col, A.n_cols, splits, part)
+        plan = HaloPlan(dA, splits, part)
         fb = S.spmv_slice_split(dA, splits, part, 1, plan.colmap, plan.S)
         hf = sp.convert(fb, "csr")
         hf.run(1.0, torch.zeros(plan.recv_len, dtype=torch.float64, device="cuda"), 1.0,
