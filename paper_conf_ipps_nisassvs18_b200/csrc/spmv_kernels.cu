@@ -572,8 +572,10 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
     }
     // rows past the window (sparse stretches: R-MAT's empty rows): the warp first writes
     // beta*y to all of them, 128 rows per step, coalesced; the tile's segments there then
-    // add alpha*s (one more rounding of beta*y than the window path, within the bound)
-    if (!ACCUM && L > kOutWin) {
+    // add alpha*s (one more rounding of beta*y than the window path, within the bound).
+    // beta == 1 leaves every row without a segment as it is: nothing to write (a halo's
+    // foreign block -- a few boundary rows in millions -- would otherwise walk them all)
+    if (!ACCUM && L > kOutWin && beta != 1.0) {
         for (int64_t g0 = Wlo + kOutWin; g0 < Whi; g0 += kOutWin) {
             double t4[kOutQ];
 #pragma unroll
@@ -1424,9 +1426,10 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
             y[lo + i] = (V)o;
         }
     }
-    if (L > kCsr5Win && moff >= 0) {
+    if (L > kCsr5Win && moff >= 0 && beta != 1.0) {
         // empty rows past the window (sparse stretches: R-MAT's empty rows) get beta*y,
         // 128 rows per step: their row pointers, then y, all loads of a step in flight
+        // (beta == 1: they stay as they are, nothing to write)
         for (int64_t g0 = lo + kCsr5Win; g0 < hi; g0 += kCsr5Win) {
             bool e[kQ];
             double t4[kQ];

@@ -105,19 +105,30 @@ def to_bytes(v, unit):
 
 
 def full(rep, out, traffic=None, formats=("coo", "ell", "csr", "hyb", "merge", "csr5")):
+    """Per launch: duration, DRAM bytes, hit rates, occupancy, registers, top stalls.  With a
+    capture taken under --nvtx (tools/prof_formats.py: one spmv_run per format inside
+    libspmv's own "spmv_run:<fmt>" ranges), every kernel of a run -- the chunk and row
+    kernels of CSR, merge's two tile kernels, the fix-ups -- is attributed to its format
+    by the range, and the traffic per run is their sum."""
     raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     r = list(csv.reader(io.StringIO(raw)))
     hdr, units = r[0], r[1]
+    nv = [h for h in hdr if h.startswith("thread Domain:Push/Pop_Range")]
     pre = "smsp__average_warps_issue_stalled_"
     lines = [f"# ncu --set full summary: {os.path.basename(rep)}\n",
-             "ncu --set full --clock-control none --import-source on (one replayed launch per row)\n",
-             "| kernel | " + " | ".join(k[1] for k in KEYS) + " | top stalls (warps per issue) |",
-             "|---|" + "---|" * (len(KEYS) + 1)]
-    seen = collections.Counter()
-    trafficmap = {}
+             "ncu --set full --clock-control none --import-source on --nvtx (one replayed launch per row; "
+             "DRAM bytes attributed to the spmv_run:<format> NVTX range each kernel ran in)\n",
+             "| range | kernel | " + " | ".join(k[1] for k in KEYS) + " | top stalls (warps per issue) |",
+             "|---|---|" + "---|" * (len(KEYS) + 1)]
+    trafficmap = collections.OrderedDict()
     for row in r[2:]:
         d = dict(zip(hdr, row))
         name = short(d["Kernel Name"])
+        rng = ""
+        if nv:
+            m = d.get(nv[0], "")
+            i = m.find("<default domain>:")
+            rng = m[i + len("<default domain>:"):].split(":none")[0] if i >= 0 else ""
         cells = []
         for k, _ in KEYS:
             u = units[hdr.index(k)] if k in hdr else ""
@@ -125,24 +136,17 @@ def full(rep, out, traffic=None, formats=("coo", "ell", "csr", "hyb", "merge", "
         st = {h[len(pre):].replace("_per_issue_active.ratio", ""): float(d[h]) for h in hdr
               if h.startswith(pre) and h.endswith("_per_issue_active.ratio") and d[h] not in ("", "n/a")}
         top = ", ".join(f"{k} {v:.1f}" for v, k in sorted(((v, k) for k, v in st.items()), reverse=True)[:3])
-        lines.append(f"| `{name}` | " + " | ".join(cells) + f" | {top} |")
-        base = name.split("<")[0]
-        seen[base] += 1
-        ta = targs(name)
-        fmt = {"k_merge": "merge", "k_merge_persist": "merge", "k_merge_rows": "merge", "k_csr5": "csr5"}.get(base)
-        if base == "k_coo":
-            fmt = "hyb" if ta[1] in ("1", "true") else "coo"
-        elif base == "k_ell":
-            fmt = "ell" if ("ell" in formats and seen[base] == 1) else "hyb"
-        elif base in ("k_csr_vector", "k_csr_rows") and seen[base] == 1 and "csr" in formats:
-            fmt = "csr"
-        elif base == "k_csr_chunks" and "csr" in formats:
-            fmt = "csr"
-        if fmt:
+        lines.append(f"| {rng} | `{name}` | " + " | ".join(cells) + f" | {top} |")
+        key = rng.replace("spmv_run:", "") if rng.startswith("spmv_run:") else ("features" if "features" in rng
+                                                                                 else None)
+        if key:
             rd = to_bytes(d["dram__bytes_read.sum"], units[hdr.index("dram__bytes_read.sum")])
             wr = to_bytes(d["dram__bytes_write.sum"], units[hdr.index("dram__bytes_write.sum")])
-            if fmt == "hyb" or fmt not in trafficmap or base == "k_csr_chunks":
-                trafficmap[fmt] = trafficmap.get(fmt, 0) + rd + wr
+            trafficmap[key] = trafficmap.get(key, 0) + rd + wr
+    if trafficmap:
+        lines += ["", "## DRAM bytes per run (all kernels of the range)", "",
+                  "| range | DRAM bytes (read+write) |", "|---|---|"]
+        lines += [f"| {k} | {v:.4g} |" for k, v in trafficmap.items()]
     with open(out, "w") as f:
         f.write("\n".join(lines) + "\n")
     print("\n".join(lines))
@@ -150,11 +154,12 @@ def full(rep, out, traffic=None, formats=("coo", "ell", "csr", "hyb", "merge", "
         cfg, dt = traffic
         p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
         d = json.load(open(p)) if os.path.exists(p) else {}
-        d.setdefault(cfg, {}).setdefault(dt, {}).update({k: int(v) for k, v in trafficmap.items()})
-        d["_note"] = ("DRAM bytes (read+write) per launch of each format's SpMV kernel, from one ncu --set full "
-                      "capture of the bench command's consistency probe (alpha=beta=1); see profiles/*.md")
+        d.setdefault(cfg, {})[dt] = {k: int(v) for k, v in trafficmap.items()}
+        d["_note"] = ("DRAM bytes (read+write) of one spmv_run of each format -- every kernel of the run, "
+                      "attributed by libspmv's spmv_run:<format> NVTX range -- and of one spmv_features call, from "
+                      "one ncu --set full --nvtx capture of tools/prof_formats.py; see profiles/*.md")
         json.dump(d, open(p, "w"), indent=1, sort_keys=True)
-        print("traffic:", trafficmap)
+        print("traffic:", dict(trafficmap))
 
 
 if __name__ == "__main__":
