@@ -147,6 +147,11 @@ typedef struct {
     int64_t csr_chunk;     /* CSR long-row split (A25): rows longer than 2*csr_chunk are cut
                               into csr_chunk-nonzero chunks, each reduced by its own warp and
                               added by the fix-up; 0 = default 512, < 0 = never split     */
+    int64_t hot_x;         /* A30 hot x columns: 0 = auto (the columns of the highest degrees,
+                              at most L2/2 worth of x entries, packed densely every run, when
+                              x exceeds twice the L2 and they hold >= 1/4 of the nonzeros),
+                              > 0 = always, at most this many columns, < 0 = never.  Not for
+                              handles that alias the input column array, nor CSR_SCALAR.  */
     const spmv_features_t *features;
                            /* optional HOST pointer: the spmv_features() result of THIS matrix
                               (same arrays, unchanged since).  The conversion then reuses it
@@ -168,6 +173,8 @@ spmv_status spmv_convert(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A,
                          const spmv_convert_opts *opts, void *stream, spmv_handle **out);
 
 /* y <- alpha*A*x + beta*y (BLAS conventions, A14): beta == 0 => y is write-only;
+ * A handle with hot columns (A30) first packs x[hot] into its own buffer (one small
+ * kernel), so one handle must not run concurrently on two streams (as for the carries); 
  * alpha == 0 => A is not read.  alpha/beta are HOST scalars of the handle's dtype
  * (float* or double*), copied at call time.  x (n_cols) and y (n_rows) are DEVICE
  * arrays of the handle's dtype; they must not overlap (SPMV_ERR_INVALID_ARG).
@@ -197,6 +204,7 @@ typedef struct {
     int64_t merge_items, merge_tiles;
     int64_t vector_width;
     int64_t csr_chunks;             /* CSR long-row chunks (A25); 0 = none */
+    int64_t hot_cols;               /* A30: hot x columns packed per run; 0 = none */
     size_t device_bytes;            /* bytes owned by the handle */
     size_t bytes_per_run;           /* algorithmic bytes of one run with beta != 0
                                        (format's own storage + x + y read + y write),
@@ -228,8 +236,11 @@ typedef enum {
     SPMV_ARR_MERGE_TILE_CLASS = 17, /* MERGE: uint8 [tiles], 1 = row-sum tile (A28): fewer than
                                        64 row ends in the tile and every row's part inside the
                                        tile (the open row included) <= 32 nonzeros; else 0     */
-    SPMV_ARR_MERGE_TILE_ORDER = 18  /* MERGE: int32 [tiles], the tile ids stably partitioned by
+    SPMV_ARR_MERGE_TILE_ORDER = 18, /* MERGE: int32 [tiles], the tile ids stably partitioned by
                                        class: class-1 tiles first (ascending), then class 0    */
+    SPMV_ARR_HOT_COLS = 19          /* any format: int32 [n_hot], the hot columns (A30), ascending;
+                                       exported column arrays are always decoded back to column
+                                       indices                                                 */
 } spmv_array_id;
 
 /* Copy array `id` of the handle to host memory (blocking on `stream`).

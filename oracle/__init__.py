@@ -92,6 +92,7 @@ def lib():
             "ora_slice_remap": (C.c_int, [_i64, _p, _p, _p, _p, C.c_int, C.c_int, _p, _p, _p]),
             "ora_partition_colmap": (_i64, [_i64, _p, _p, _p, C.c_int, _p]),
             "ora_halo_colmap": (_i64, [_i64, _p, _p, _p, C.c_int, C.c_int, _p, _p]),
+            "ora_hot_columns": (_i64, [_i64, _i64, _p, _i64, _p]),
             "ora_slice_remap_colmap": (C.c_int, [_i64, _p, _p, _p, _p, C.c_int, _p, _p, _p, _p]),
             "ora_slice_split": (_i64, [_i64, _p, _p, _p, _p, C.c_int, C.c_int, _p, C.c_int, _p, _p, _p]),
         }
@@ -335,6 +336,16 @@ def partition_colmap(A, splits):
     S = lib().ora_partition_colmap(A.n_rows, _ptr(A.row_ptr), _ptr(A.col), _ptr(s), s.size - 1, _ptr(cm))
     assert S >= 0
     return cm, int(S)
+
+
+def hot_columns(A, kmax):
+    """A30: the hot x columns of A for a budget of kmax columns (ascending int32)."""
+    A = CSR.of(A)
+    K = lib().ora_hot_columns(A.n_cols, A.nnz, _ptr(A.col), int(kmax), None)
+    assert K >= 0
+    out = _buf(K, np.int32)
+    lib().ora_hot_columns(A.n_cols, A.nnz, _ptr(A.col), int(kmax), _ptr(out))
+    return out
 
 
 def halo_colmap(A, splits, part):

@@ -602,6 +602,31 @@ int64_t ora_partition_colmap(int64_t n_rows, const int64_t *row_ptr, const int32
     return S;
 }
 
+/* A30 hot columns (a handle's x layout): the degree of column c is its
+ * number of nonzeros; the hot set is every column of degree >= t for the smallest t >= 1
+ * such that at most kmax columns qualify, listed ascending.  Plain loops: degrees, a
+ * count per degree value, then t.  Returns the number of hot columns (hot_out may be NULL). */
+int64_t ora_hot_columns(int64_t n_cols, int64_t nnz, const int32_t *col, int64_t kmax, int32_t *hot_out)
+{
+    if (n_cols <= 0 || nnz <= 0 || kmax <= 0) return 0;
+    int64_t *deg = (int64_t *)calloc((size_t)n_cols, sizeof(int64_t));
+    if (!deg) return -1;
+    int64_t dmax = 0;
+    for (int64_t k = 0; k < nnz; ++k) deg[col[k]] += 1;
+    for (int64_t c = 0; c < n_cols; ++c) if (deg[c] > dmax) dmax = deg[c];
+    int64_t *cnt = (int64_t *)calloc((size_t)dmax + 2, sizeof(int64_t));     /* cnt[v] = #{deg == v} */
+    if (!cnt) { free(deg); return -1; }
+    for (int64_t c = 0; c < n_cols; ++c) cnt[deg[c]] += 1;
+    int64_t t = dmax + 1, ge = 0;                                         /* ge = #{deg >= t} */
+    while (t > 1 && ge + cnt[t - 1] <= kmax) { t -= 1; ge += cnt[t]; }
+    int64_t K = 0;
+    for (int64_t c = 0; c < n_cols; ++c)
+        if (deg[c] >= t) { if (hot_out) hot_out[K] = (int32_t)c; ++K; }
+    free(cnt);
+    free(deg);
+    return K;
+}
+
 /* Halo exchange: receiver `part` needs the columns its rows reference
  * that other parts own.  Plain loops: mark them, count per owner, S = max(1, max count),
  * colmap[j] = owner*S + (rank of j among the owner's marked columns), -1 elsewhere.

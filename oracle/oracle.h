@@ -149,6 +149,7 @@ int ora_slice_remap(int64_t n_rows, const int64_t *row_ptr, const int32_t *col,
 /* Compressed exchange: colmap[j] = owner(j)*S' + (referenced columns of
  * owner(j) before j) for a column some row references, -1 otherwise; returns S' (max
  * referenced columns per part).  Square matrices. */
+int64_t ora_hot_columns(int64_t n_cols, int64_t nnz, const int32_t *col, int64_t kmax, int32_t *hot_out);
 int64_t ora_halo_colmap(int64_t n_rows, const int64_t *row_ptr, const int32_t *col, const int64_t *splits,
                         int nparts, int part, int32_t *colmap, int64_t *counts);
 int64_t ora_partition_colmap(int64_t n_rows, const int64_t *row_ptr, const int32_t *col,

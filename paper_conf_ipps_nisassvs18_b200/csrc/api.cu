@@ -2,6 +2,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <vector>
 
 #include <nvtx3/nvToolsExt.h>
 
@@ -280,6 +281,7 @@ spmv_status spmv_info(const spmv_handle *h, spmv_handle_info *o) {
     o->merge_tiles = h->merge_tiles;
     o->vector_width = h->vec_w;
     o->csr_chunks = h->csr_chunks;
+    o->hot_cols = h->n_hot;
     size_t dev = 0, fmt_bytes = 0;
     for (int i = 0; i < kMaxArrays; ++i) {
         if (h->arr[i].owned) dev += h->arr[i].bytes;
@@ -287,13 +289,16 @@ spmv_status spmv_info(const spmv_handle *h, spmv_handle_info *o) {
         // class from the tile order: both kept for export, not read by a run
         if (i != SPMV_ARR_MERGE_COORD_NZ && i != SPMV_ARR_MERGE_TILE_CLASS) fmt_bytes += h->arr[i].bytes;
     }
-    dev += h->carry_row.bytes + h->carry_val.bytes + h->sched.bytes;
+    dev += h->carry_row.bytes + h->carry_val.bytes + h->sched.bytes + h->xhot.bytes;
     o->device_bytes = dev;
     // algorithmic bytes per run: the format's own arrays + x + y
     size_t V = h->dtype == SPMV_F64 ? 8 : 4;
     size_t xy = (size_t)h->n_cols * V + (size_t)h->n_rows * V;
-    o->bytes_per_run_beta0 = fmt_bytes + xy;
-    o->bytes_per_run = fmt_bytes + xy + (size_t)h->n_rows * V;
+    // A30: the per-run hot pack reads x[hot] (counted in x), writes xhot, the kernels read it
+    // back; the hot-column list itself is counted with the format's arrays
+    const size_t hot = (size_t)h->n_hot * V * 2;
+    o->bytes_per_run_beta0 = fmt_bytes + xy + hot;
+    o->bytes_per_run = fmt_bytes + xy + hot + (size_t)h->n_rows * V;
     return SPMV_OK;
 }
 
@@ -318,6 +323,7 @@ spmv_status spmv_export(const spmv_handle *h, spmv_array_id id, void *dst, size_
                                    id == SPMV_ARR_MERGE_TILE_ORDER; break;
         case SPMV_CSR5: present = id <= SPMV_ARR_VAL || (id >= SPMV_ARR_CSR5_TILE_PTR && id <= SPMV_ARR_CSR5_SEG_MAP); break;
         }
+        if (id == SPMV_ARR_HOT_COLS) present = true;            // A30: empty when no hot columns
         if (!present) { set_error("handle has no such array"); return SPMV_ERR_INVALID_ARG; }
         return SPMV_OK;
     }
@@ -326,6 +332,16 @@ spmv_status spmv_export(const spmv_handle *h, spmv_array_id id, void *dst, size_
     SPMV_ON_DEVICE(h->ctx->device);
     SPMV_CUDA_TRY(cudaMemcpyAsync(dst, a.p, a.bytes, cudaMemcpyDeviceToHost, s));
     SPMV_CUDA_TRY(cudaStreamSynchronize(s));
+    if (h->n_hot > 0 && (id == SPMV_ARR_COL || id == SPMV_ARR_ELL_COL || id == SPMV_ARR_HYB_COO_COL)) {
+        // A30: column arrays are exported as column indices (-2 - slot -> hot[slot])
+        std::vector<int32_t> hot((size_t)h->n_hot);
+        SPMV_CUDA_TRY(cudaMemcpyAsync(hot.data(), h->arr[SPMV_ARR_HOT_COLS].p, hot.size() * 4,
+                                      cudaMemcpyDeviceToHost, s));
+        SPMV_CUDA_TRY(cudaStreamSynchronize(s));
+        int32_t *c = static_cast<int32_t *>(dst);
+        for (size_t k = 0; k < a.bytes / 4; ++k)
+            if (c[k] <= -2) c[k] = hot[(size_t)(-2 - c[k])];
+    }
     return SPMV_OK;
 }
 
@@ -339,6 +355,7 @@ spmv_status spmv_destroy(spmv_handle *h, void *stream) {
     dev_free(h->ctx, h->carry_val.p, h->carry_val.bytes, s);
     dev_free(h->ctx, h->io_x.p, h->io_x.bytes, s);
     dev_free(h->ctx, h->sched.p, h->sched.bytes, s);
+    dev_free(h->ctx, h->xhot.p, h->xhot.bytes, s);
     dev_free(h->ctx, h->io_y.p, h->io_y.bytes, s);
     delete h;
     return SPMV_OK;

@@ -146,6 +146,15 @@ __device__ __forceinline__ int ld_x(const int *p, uint64_t pol) {
     return v;
 }
 
+// A30 hot columns: a handle may store the column of a hot x entry as -2 - slot (-1 stays
+// the "no element" sentinel of ELL padding and partial loads); its value is then
+// xh[slot], the run's densely packed copy of the hot x entries
+template <bool HOT, typename V>
+__device__ __forceinline__ const V *xp(const V *x, const V *xh, int c) {
+    if constexpr (HOT) return c >= 0 ? x + c : xh + (-2 - c);
+    else return x + c;
+}
+
 // plain read-only loads for metadata (row_ptr, descriptors)
 template <typename T> __device__ __forceinline__ T ldg(const T *p) { return __ldg(p); }
 

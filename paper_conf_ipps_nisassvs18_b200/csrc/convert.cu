@@ -597,12 +597,23 @@ spmv_status convert_impl(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, cons
         return SPMV_ERR_NOT_CANONICAL;
     }
     const bool i64 = A->nnz > INT32_MAX || o->index64;
+    spmv_status st;
     if (A->dtype == SPMV_F64) {
-        return i64 ? convert_t<int64_t, double>(ctx, fmt, A, o, s, h, fs, cusp)
-                   : convert_t<int, double>(ctx, fmt, A, o, s, h, fs, cusp);
+        st = i64 ? convert_t<int64_t, double>(ctx, fmt, A, o, s, h, fs, cusp)
+                 : convert_t<int, double>(ctx, fmt, A, o, s, h, fs, cusp);
+    } else {
+        st = i64 ? convert_t<int64_t, float>(ctx, fmt, A, o, s, h, fs, cusp)
+                 : convert_t<int, float>(ctx, fmt, A, o, s, h, fs, cusp);
     }
-    return i64 ? convert_t<int64_t, float>(ctx, fmt, A, o, s, h, fs, cusp)
-               : convert_t<int, float>(ctx, fmt, A, o, s, h, fs, cusp);
+    if (st != SPMV_OK || o->hot_x < 0 || fmt == SPMV_CSR_SCALAR) return st;
+    // A30: hot x columns packed densely -- only where the handle owns its column arrays
+    for (int id : {(int)SPMV_ARR_COL, (int)SPMV_ARR_ELL_COL, (int)SPMV_ARR_HYB_COO_COL})
+        if (h->arr[id].p && !h->arr[id].owned) return SPMV_OK;
+    const size_t V = A->dtype == SPMV_F64 ? 8 : 4;
+    const int64_t kmax = o->hot_x > 0 ? o->hot_x : (int64_t)(ctx->l2_bytes / 2 / V);
+    Scratch slot(ctx, s);
+    SPMV_TRY(hot_select(ctx, A, kmax, o->hot_x > 0, s, h, slot));
+    return hot_encode(ctx, h, slot, s);
 }
 
 }  // namespace spmv

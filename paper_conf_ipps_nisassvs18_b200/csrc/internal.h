@@ -19,7 +19,7 @@ struct spmv_ctx {
 
 namespace spmv {
 
-constexpr int kMaxArrays = 19;
+constexpr int kMaxArrays = 20;
 
 struct DevArray {
     void *p = nullptr;
@@ -90,6 +90,10 @@ struct spmv_handle {
     spmv::DevArray io_x, io_y;
     // CSR-vector dynamic batch scheduler: one u64 counter, zeroed before every run
     spmv::DevArray sched;
+    // hot columns (A30): the x entries stored as -2 - slot are read from xhot[slot], packed
+    // from x[arr[SPMV_ARR_HOT_COLS][slot]] at the start of every run (n_hot = 0: none)
+    spmv::DevArray xhot;
+    int64_t n_hot = 0;
     int launches = 0;
 };
 
@@ -97,6 +101,10 @@ namespace spmv {
 // convert.cu
 spmv_status convert_impl(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A,
                          const spmv_convert_opts *opts, cudaStream_t s, spmv_handle *h);
+// hot.cu (A30)
+spmv_status hot_select(spmv_ctx *ctx, const spmv_csr *A, int64_t kmax, bool force, cudaStream_t s,
+                       spmv_handle *h, Scratch &slot);
+spmv_status hot_encode(spmv_ctx *ctx, spmv_handle *h, const Scratch &slot, cudaStream_t s);
 // spmv_kernels.cu
 spmv_status run_impl(spmv_handle *h, double alpha, double beta, const void *x, void *y,
                      cudaStream_t s);

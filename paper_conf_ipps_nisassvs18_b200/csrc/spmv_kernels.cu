@@ -58,6 +58,14 @@ __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.lau
 
 // ------------------------------------------------------------------ alpha == 0
 
+// A30: xh[i] = x[hot[i]] -- the run's values of the handle's hot columns, packed densely
+// so that the gathers to them hit L2 (and L1) four (fp64) / eight (fp32) per sector
+template <typename V>
+__global__ void k_hot_gather(const V *__restrict__ x, const int *__restrict__ hot, int64_t k, V *__restrict__ xh) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < k; i += (int64_t)gridDim.x * blockDim.x)
+        xh[i] = __ldg(x + __ldg(hot + i));
+}
+
 template <typename V, bool B0>
 __global__ void k_scale(V *y, int64_t n, double beta) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
@@ -75,10 +83,10 @@ __global__ void k_scale(V *y, int64_t n, double beta) {
 // folded every kFold steps, A13) -- the paper's warp-per-row kernel for long rows.
 template <int W> struct VecCfg { static constexpr int U = W <= 8 ? 32 / (32 / W) : (W == 16 ? 4 : 2); };
 
-template <typename V, typename IT, int W, bool B0, int MB, bool CHUNKED, bool DYN = false>
+template <typename V, typename IT, int W, bool B0, int MB, bool CHUNKED, bool DYN = false, bool HOT = false>
 __global__ void __launch_bounds__(kT, MB)
 k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
-             const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta, int64_t long_len,
+             const V *__restrict__ x, const V *__restrict__ xh, V *__restrict__ y, int64_t n, double alpha, double beta, int64_t long_len,
              unsigned long long *__restrict__ sched = nullptr) {
     constexpr int G = 32 / W;
     constexpr int U = (VecCfg<W>::U * G > 32) ? 32 / G : VecCfg<W>::U;
@@ -158,7 +166,7 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
         }
         double s[U];
 #pragma unroll
-        for (int u = 0; u < U; ++u) s[u] = c0[u] >= 0 ? (double)v0[u] * (double)ld_x(x + c0[u], px) : 0.0;
+        for (int u = 0; u < U; ++u) s[u] = c0[u] != -1 ? (double)v0[u] * (double)ld_x(xp<HOT>(x, xh, c0[u]), px) : 0.0;
         // the group's U results: lane sub == u of group g writes row u*G + g
         double mine = 0.0;
         {
@@ -221,7 +229,7 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
                         w[q] = in ? ld_hint(val + k + q * SW, pa) : (V)0;
                     }
 #pragma unroll
-                    for (int q = 0; q < 8; ++q) if (d[q] >= 0) acc[q] += (double)w[q] * (double)ld_x(x + d[q], px);
+                    for (int q = 0; q < 8; ++q) if (d[q] != -1) acc[q] += (double)w[q] * (double)ld_x(xp<HOT>(x, xh, d[q]), px);
                 }
                 double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
                 for (int o = SW >> 1; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
@@ -247,14 +255,14 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
 #pragma unroll
                     for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
 #pragma unroll
-                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(x + d[q], px);
+                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(xp<HOT>(x, xh, d[q]), px);
                     if (++it == kFold) {                 // blocked summation (A13)
 #pragma unroll
                         for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
                         it = 0;
                     }
                 }
-                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
+                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(xp<HOT>(x, xh, ld_hint(col + k, pa)), px);
                 double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
                 part = warp_sum(tot + part);
                 const int writer = (i / U) * W + i % U;   // lane holding row i's group sum
@@ -278,11 +286,11 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
 // One warp per C-nonzero chunk of a long row (8 loads per lane in flight, blocked
 // summation, A13); the chunk sum is the carry (row, value) that the fix-up adds in
 // chunk order.  The row-batch kernel wrote beta*y for these rows.
-template <typename V, typename IT>
+template <typename V, typename IT, bool HOT = false>
 __global__ void __launch_bounds__(kT)
 k_csr_chunks(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
              const int64_t *__restrict__ crow, const int64_t *__restrict__ clo, int64_t nch, int64_t C,
-             const V *__restrict__ x, int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
+             const V *__restrict__ x, const V *__restrict__ xh, int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
     pdl_trigger();
     const int lane = threadIdx.x & 31;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
@@ -302,14 +310,14 @@ k_csr_chunks(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
 #pragma unroll
             for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
 #pragma unroll
-            for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(x + d[q], px);
+            for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(xp<HOT>(x, xh, d[q]), px);
             if (++it == kFold) {
 #pragma unroll
                 for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
                 it = 0;
             }
         }
-        for (; k < hi; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
+        for (; k < hi; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(xp<HOT>(x, xh, ld_hint(col + k, pa)), px);
         const double part = warp_sum(tot + (((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]))));
         if (lane == 0) { carry_row[c] = r; carry_val[c] = part; }
     }
@@ -317,20 +325,20 @@ k_csr_chunks(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
 
 // ------------------------------------------------------------------ CSR-scalar (K2)
 // "assigning a thread to process each row -- the scalar CSR kernel".
-template <typename V, typename IT, bool B0>
+template <typename V, typename IT, bool B0, bool HOT = false>
 __global__ void __launch_bounds__(kT)
 k_csr_scalar(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
-             const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta) {
+             const V *__restrict__ x, const V *__restrict__ xh, V *__restrict__ y, int64_t n, double alpha, double beta) {
     const uint64_t px = policy_evict_last();
     for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
         const double yv = B0 ? 0.0 : (double)y[r];
         double a0 = 0.0, a1 = 0.0;
         int64_t k = __ldg(rp + r), b = __ldg(rp + r + 1);
         for (; k + 1 < b; k += 2) {
-            a0 += (double)__ldg(val + k) * (double)ld_x(x + __ldg(col + k), px);
-            a1 += (double)__ldg(val + k + 1) * (double)ld_x(x + __ldg(col + k + 1), px);
+            a0 += (double)__ldg(val + k) * (double)ld_x(xp<HOT>(x, xh, __ldg(col + k)), px);
+            a1 += (double)__ldg(val + k + 1) * (double)ld_x(xp<HOT>(x, xh, __ldg(col + k + 1)), px);
         }
-        if (k < b) a0 += (double)__ldg(val + k) * (double)ld_x(x + __ldg(col + k), px);
+        if (k < b) a0 += (double)__ldg(val + k) * (double)ld_x(xp<HOT>(x, xh, __ldg(col + k)), px);
         double o = alpha * (a0 + a1);
         if (!B0) o = fma(beta, yv, o);
         y[r] = (V)o;
@@ -374,10 +382,10 @@ template <typename V> __device__ __forceinline__ V lane_of(const V &v, int) { re
 __device__ __forceinline__ double lane_of(const double2 &v, int r) { return r ? v.y : v.x; }
 __device__ __forceinline__ float lane_of(const float2 &v, int r) { return r ? v.y : v.x; }
 
-template <typename V, bool B0, int RPT, int BATCH>
+template <typename V, bool B0, int RPT, int BATCH, bool HOT = false>
 __global__ void __launch_bounds__(kT)
 k_ell(const int *__restrict__ ecol, const V *__restrict__ eval, int64_t K, int64_t ld,
-      const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta) {
+      const V *__restrict__ x, const V *__restrict__ xh, V *__restrict__ y, int64_t n, double alpha, double beta) {
     using CT = typename EllVec<V, RPT>::CT;
     using VT = typename EllVec<V, RPT>::VT;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
@@ -412,10 +420,10 @@ k_ell(const int *__restrict__ ecol, const V *__restrict__ eval, int64_t K, int64
 #pragma unroll
                 for (int u = 0; u < BATCH; u += 2) {
                     const int cu = lane_of(c[u], q);
-                    if (j0 + u < K && cu >= 0) a0 += (double)lane_of(v[u], q) * (double)ld_x(x + cu, px);
+                    if (j0 + u < K && cu != -1) a0 += (double)lane_of(v[u], q) * (double)ld_x(xp<HOT>(x, xh, cu), px);
                     if (u + 1 < BATCH) {
                         const int cw = lane_of(c[u + 1], q);
-                        if (j0 + u + 1 < K && cw >= 0) a1 += (double)lane_of(v[u + 1], q) * (double)ld_x(x + cw, px);
+                        if (j0 + u + 1 < K && cw != -1) a1 += (double)lane_of(v[u + 1], q) * (double)ld_x(xp<HOT>(x, xh, cw), px);
                     }
                 }
                 part[q] += a0 + a1;
@@ -502,10 +510,10 @@ template <> struct VecLoad8<float> {
 };
 __device__ __forceinline__ void load_int8(const int *p, int (&v)[8], uint64_t pol) { ld256(p, v, pol); }
 
-template <typename V, bool ACCUM, bool B0>
+template <typename V, bool ACCUM, bool B0, bool HOT = false>
 __global__ void __launch_bounds__(kT, kMinBlocks)
 k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restrict__ val, int64_t nnz,
-      int64_t n_tiles, const V *__restrict__ x, V *__restrict__ y, int64_t n_rows, double alpha, double beta,
+      int64_t n_tiles, const V *__restrict__ x, const V *__restrict__ xh, V *__restrict__ y, int64_t n_rows, double alpha, double beta,
       int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
     static_assert(kWIPT == 8, "COO lane chunk is 8 elements");
     __shared__ double s_acc_all[kT / 32][kOutWin];
@@ -540,7 +548,7 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
     double p[8];
     if constexpr (sizeof(V) == 4) {
 #pragma unroll
-        for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
+        for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(xp<HOT>(x, xh, c[s]), px) : 0.0;
     }
     // rows around the tile (uniform loads)
     const int rf = __shfl_sync(0xffffffffu, r[0], 0);                       // tile's first row
@@ -568,7 +576,7 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
     }
     if constexpr (sizeof(V) == 8) {
 #pragma unroll
-        for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(x + c[s], px) : 0.0;
+        for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(xp<HOT>(x, xh, c[s]), px) : 0.0;
     }
     // rows past the window (sparse stretches: R-MAT's empty rows): the warp first writes
     // beta*y to all of them, 128 rows per step, coalesced; the tile's segments there then
@@ -647,8 +655,8 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
 // [st, st + len) of one row, 8 slots per step with all x gathers of a step in flight.
 // Called by all lanes with their own row, so at slot j the warp gathers x for
 // consecutive rows (few L1 wavefronts on banded matrices, as ELL).
-template <typename V>
-__device__ __forceinline__ double row_walk(const int *s_c, const V *s_v, int st, int len, const V *__restrict__ x,
+template <typename V, bool HOT = false>
+__device__ __forceinline__ double row_walk(const int *s_c, const V *s_v, int st, int len, const V *__restrict__ x, const V *__restrict__ xh,
                                            uint64_t px) {
     double a0 = 0.0, a1 = 0.0;
     for (int k = 0; k < len; k += 8) {
@@ -662,7 +670,7 @@ __device__ __forceinline__ double row_walk(const int *s_c, const V *s_v, int st,
         }
         double pp[8];
 #pragma unroll
-        for (int u = 0; u < 8; ++u) pp[u] = k + u < len ? (double)vv[u] * (double)ld_x(x + cc[u], px) : 0.0;
+        for (int u = 0; u < 8; ++u) pp[u] = k + u < len ? (double)vv[u] * (double)ld_x(xp<HOT>(x, xh, cc[u]), px) : 0.0;
 #pragma unroll
         for (int u = 0; u < 8; u += 2) { a0 += pp[u]; a1 += pp[u + 1]; }
     }
@@ -670,9 +678,9 @@ __device__ __forceinline__ double row_walk(const int *s_c, const V *s_v, int st,
 }
 // the same walk reading col/val from global memory (rows of a batch that does not fit
 // the shared-memory chunk)
-template <typename V>
+template <typename V, bool HOT = false>
 __device__ __forceinline__ double row_walk_global(const int *__restrict__ col, const V *__restrict__ val, int64_t a,
-                                                  int len, const V *__restrict__ x, uint64_t pa, uint64_t px) {
+                                                  int len, const V *__restrict__ x, const V *__restrict__ xh, uint64_t pa, uint64_t px) {
     double a0 = 0.0, a1 = 0.0;
     for (int k = 0; k < len; k += 8) {
         int cc[8];
@@ -685,7 +693,7 @@ __device__ __forceinline__ double row_walk_global(const int *__restrict__ col, c
         }
         double pp[8];
 #pragma unroll
-        for (int u = 0; u < 8; ++u) pp[u] = k + u < len ? (double)vv[u] * (double)ld_x(x + cc[u], px) : 0.0;
+        for (int u = 0; u < 8; ++u) pp[u] = k + u < len ? (double)vv[u] * (double)ld_x(xp<HOT>(x, xh, cc[u]), px) : 0.0;
 #pragma unroll
         for (int u = 0; u < 8; u += 2) { a0 += pp[u]; a1 += pp[u + 1]; }
     }
@@ -737,10 +745,10 @@ __device__ __forceinline__ void chunk_store(int *s_c, V *s_v, int pos, const int
 // all) is reduced row by row by the whole warp (the paper's warp-per-row vector
 // kernel; blocked summation, A13).  CHUNKED: rows longer than long_len
 // get beta*y here and their chunks arrive through the fix-up (A25).
-template <typename V, typename IT, bool B0, int MB, bool CHUNKED>
+template <typename V, typename IT, bool B0, int MB, bool CHUNKED, bool HOT = false>
 __global__ void __launch_bounds__(kT, MB)
 k_csr_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
-           const V *__restrict__ x, V *__restrict__ y, int64_t n, double alpha, double beta, int64_t long_len) {
+           const V *__restrict__ x, const V *__restrict__ xh, V *__restrict__ y, int64_t n, double alpha, double beta, int64_t long_len) {
     __shared__ __align__(16) double s_p_all[kT / 32][264 + 132];   // values, then cols
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     double *s_p = s_p_all[wid];
@@ -786,7 +794,7 @@ k_csr_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
             __syncwarp();
             int len = (int)(my_e - my_a);
             if (CHUNKED && len > long_len) len = 0;            // A25: chunks via the fix-up
-            sum = row_walk(s_c, s_v, (int)(my_a - lo) + off, len, x, px);
+            sum = row_walk<V, HOT>(s_c, s_v, (int)(my_a - lo) + off, len, x, xh, px);
             __syncwarp();
         } else {
             // rows <= 32 nonzeros: lane i walks row b + i straight from global memory;
@@ -794,7 +802,7 @@ k_csr_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
             int64_t len = my_e - my_a;
             if (CHUNKED && len > long_len) len = 0;            // A25: chunks via the fix-up
             const bool lng = len > 32;
-            if (!lng) sum = row_walk_global(col, val, my_a, (int)len, x, pa, px);
+            if (!lng) sum = row_walk_global<V, HOT>(col, val, my_a, (int)len, x, xh, pa, px);
             unsigned lm = __ballot_sync(0xffffffffu, lng);
             while (lm) {
                 const int i = __ffs(lm) - 1;
@@ -811,14 +819,14 @@ k_csr_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
 #pragma unroll
                     for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
 #pragma unroll
-                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(x + d[q], px);
+                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(xp<HOT>(x, xh, d[q]), px);
                     if (++it == kFold) {
 #pragma unroll
                         for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
                         it = 0;
                     }
                 }
-                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(x + ld_hint(col + k, pa), px);
+                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(xp<HOT>(x, xh, ld_hint(col + k, pa)), px);
                 const double part = warp_sum(tot + (((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]))));
                 if (lane == i) sum = part;
             }
@@ -889,10 +897,10 @@ template <int N> struct ShiftLoad<int, N> {
     static __device__ __forceinline__ void load(const int *p, int (&v)[N], uint64_t pol) { shift_load4<int, int4, N>(p, v, pol); }
 };
 
-template <typename V, typename IT, bool B0, int LI>
+template <typename V, typename IT, bool B0, int LI, bool HOT = false>
 __device__ __forceinline__ void
 merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val, int64_t t,
-           int64_t r0, int64_t r1, int64_t k0, int64_t k1, const V *__restrict__ x, V *__restrict__ y,
+           int64_t r0, int64_t r1, int64_t k0, int64_t k1, const V *__restrict__ x, const V *__restrict__ xh, V *__restrict__ y,
            double alpha, double beta, int64_t *__restrict__ carry_row, double *__restrict__ carry_val,
            double *s_sum, int *s_end, uint2 *s_flag, uint64_t pa, uint64_t px) {
     constexpr int TI = 32 * LI;
@@ -931,7 +939,7 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
     double p[LI];
 #pragma unroll
     for (int e = 0; e < LI; ++e)
-        p[e] = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)v[e] * (double)ld_x(x + c[e], px) : 0.0;
+        p[e] = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)v[e] * (double)ld_x(xp<HOT>(x, xh, c[e]), px) : 0.0;
     __syncwarp();
     // segment starts: local row i (1 <= i <= nrows) starts at s_end[i-1]; row 0 at 0 if
     // r0_inside.  The bitmap is indexed by chunk position (tile position + off).
@@ -984,7 +992,7 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
                     cur = pos;
                     acc = 0.0;
                 }
-                acc += (double)ld_hint(val + k0 + pos, pa) * (double)ld_x(x + ld_hint(col + k0 + pos, pa), px);
+                acc += (double)ld_hint(val + k0 + pos, pa) * (double)ld_x(xp<HOT>(x, xh, ld_hint(col + k0 + pos, pa)), px);
             }
         }
     }
@@ -1034,11 +1042,11 @@ __device__ __forceinline__ int64_t merge_k(int64_t t, int TI, int64_t r, int64_t
 }
 
 // one warp per tile
-template <typename V, typename IT, bool B0, int LI, int MB = kMinBlocks>
+template <typename V, typename IT, bool B0, int LI, int MB = kMinBlocks, bool HOT = false>
 __global__ void __launch_bounds__(kT, MB)
 k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
         const int64_t *__restrict__ crow, int64_t n_tiles, int64_t dmax,
-        const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
+        const V *__restrict__ x, const V *__restrict__ xh, V *__restrict__ y, double alpha, double beta,
         int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
     constexpr int TI = 32 * LI;
     __shared__ double s_sum_all[kT / 32][TI];             // segment sum, keyed by its start position
@@ -1049,7 +1057,7 @@ k_merge(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restr
     if (t >= n_tiles) return;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
     const int64_t r0 = ld_coord(crow + t, px), r1 = ld_coord(crow + t + 1, px);
-    merge_tile<V, IT, B0, LI>(rp, col, val, t, r0, r1, merge_k(t, TI, r0, dmax), merge_k(t + 1, TI, r1, dmax), x, y,
+    merge_tile<V, IT, B0, LI, HOT>(rp, col, val, t, r0, r1, merge_k(t, TI, r0, dmax), merge_k(t + 1, TI, r1, dmax), x, xh, y,
                               alpha, beta, carry_row, carry_val, s_sum_all[wid], s_end_all[wid], s_flag_all[wid], pa,
                               px);
 }
@@ -1091,11 +1099,11 @@ __device__ __forceinline__ int64_t ld_rp(const int64_t *p) {
 // Segmented-sum tiles (any class).  LIST = false: tiles i0 + w, i0 + w + W, ... (the
 // next tile's coordinates loaded while the current one runs); LIST = true: positions
 // [i0, i1) of the tile order.
-template <typename V, typename IT, bool B0, int LI, int MB, bool LIST>
+template <typename V, typename IT, bool B0, int LI, int MB, bool LIST, bool HOT = false>
 __global__ void __launch_bounds__(kT, MB)
 k_merge_persist(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
                 const int64_t *__restrict__ crow, const int *__restrict__ order, int64_t i0, int64_t i1,
-                int64_t dmax, const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
+                int64_t dmax, const V *__restrict__ x, const V *__restrict__ xh, V *__restrict__ y, double alpha, double beta,
                 int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
     constexpr int TI = 32 * LI;
     __shared__ double s_sum_all[kT / 32][TI];
@@ -1104,7 +1112,7 @@ k_merge_persist(const IT *__restrict__ rp, const int *__restrict__ col, const V 
     const int wid = threadIdx.x >> 5;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
     auto body = [&](int64_t t, int64_t r0, int64_t r1) {
-        merge_tile<V, IT, B0, LI>(rp, col, val, t, r0, r1, merge_k(t, TI, r0, dmax), merge_k(t + 1, TI, r1, dmax), x, y,
+        merge_tile<V, IT, B0, LI, HOT>(rp, col, val, t, r0, r1, merge_k(t, TI, r0, dmax), merge_k(t + 1, TI, r1, dmax), x, xh, y,
                                   alpha, beta, carry_row, carry_val, s_sum_all[wid], s_end_all[wid], s_flag_all[wid],
                                   pa, px);
     };
@@ -1178,10 +1186,10 @@ __device__ __forceinline__ void merge_chunk_load(const int *__restrict__ col, co
     }
 }
 
-template <typename V, typename IT, bool B0, bool PAIRS>
+template <typename V, typename IT, bool B0, bool PAIRS, bool HOT = false>
 __device__ __forceinline__ void
 merge_rows_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val, int64_t t,
-                int64_t r0, int64_t r1, int64_t k0, int64_t k1, const MergeChunk<V> &ch, const V *__restrict__ x,
+                int64_t r0, int64_t r1, int64_t k0, int64_t k1, const MergeChunk<V> &ch, const V *__restrict__ x, const V *__restrict__ xh,
                 V *__restrict__ y, double alpha, double beta, int64_t *__restrict__ carry_row,
                 double *__restrict__ carry_val, double *s_p, uint64_t pa, uint64_t px) {
     constexpr int LI = 8;
@@ -1208,14 +1216,14 @@ merge_rows_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V 
 #pragma unroll
     for (int e = 0; e < LI; e += 2) {
         const int pe = chunk_pos<V, PAIRS>(lane, e);      // chunk position of element e (pe + 1 of e + 1)
-        const double p0 = (ends_in && (unsigned)(pe - off) < (unsigned)nnzt) ? (double)ch.v[e] * (double)ld_x(x + ch.c[e], px) : 0.0;
-        const double p1 = (ends_in && (unsigned)(pe + 1 - off) < (unsigned)nnzt) ? (double)ch.v[e + 1] * (double)ld_x(x + ch.c[e + 1], px) : 0.0;
+        const double p0 = (ends_in && (unsigned)(pe - off) < (unsigned)nnzt) ? (double)ch.v[e] * (double)ld_x(xp<HOT>(x, xh, ch.c[e]), px) : 0.0;
+        const double p1 = (ends_in && (unsigned)(pe + 1 - off) < (unsigned)nnzt) ? (double)ch.v[e + 1] * (double)ld_x(xp<HOT>(x, xh, ch.c[e + 1]), px) : 0.0;
         *reinterpret_cast<double2 *>(s_p + pe) = make_double2(p0, p1);
     }
     if (lane == 31) {                                     // positions past lane 31's chunk (< off row ends)
 #pragma unroll 1
         for (int pos = j0 + LI; pos < nnzt; ++pos)
-            s_p[pos + off] = (double)ld_hint(val + k0 + pos, pa) * (double)ld_x(x + ld_hint(col + k0 + pos, pa), px);
+            s_p[pos + off] = (double)ld_hint(val + k0 + pos, pa) * (double)ld_x(xp<HOT>(x, xh, ld_hint(col + k0 + pos, pa)), px);
     }
     int s0 = __shfl_up_sync(0xffffffffu, e_[0], 1);
     const int last0 = __shfl_sync(0xffffffffu, e_[0], 31);
@@ -1248,11 +1256,11 @@ merge_rows_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V 
 // takes tiles w, w + W, ... and the next tile's coordinates are loaded while the current
 // one runs; LIST = true: positions [i0, i1) of the tile order (SPMV_MERGE_SCHEDULE).
 // The identity schedule is measurably faster than the list (LAP4096: 0.298 vs 0.339 ms).
-template <typename V, typename IT, bool B0, int MB, bool LIST, bool PAIRS = true>
+template <typename V, typename IT, bool B0, int MB, bool LIST, bool PAIRS = true, bool HOT = false>
 __global__ void __launch_bounds__(kT, MB)
 k_merge_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
              const int64_t *__restrict__ crow, const int *__restrict__ order, int64_t i0, int64_t i1,
-             int64_t dmax, const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
+             int64_t dmax, const V *__restrict__ x, const V *__restrict__ xh, V *__restrict__ y, double alpha, double beta,
              int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
     __shared__ __align__(16) double s_p_all[kT / 32][256 + 8];
     const int wid = threadIdx.x >> 5;
@@ -1261,7 +1269,7 @@ k_merge_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
         MergeChunk<V> ch;
         const int64_t k0 = merge_k(t, 256, r0, dmax), k1 = merge_k(t + 1, 256, r1, dmax);
         merge_chunk_load<V, PAIRS>(col, val, k0, k1, ch, pa);
-        merge_rows_tile<V, IT, B0, PAIRS>(rp, col, val, t, r0, r1, k0, k1, ch, x, y, alpha, beta, carry_row, carry_val,
+        merge_rows_tile<V, IT, B0, PAIRS, HOT>(rp, col, val, t, r0, r1, k0, k1, ch, x, xh, y, alpha, beta, carry_row, carry_val,
                                    s_p_all[wid], pa, px);
     };
     if constexpr (!LIST) {
@@ -1322,13 +1330,13 @@ struct Csr5Vec<SIGMA, float> {
     }
 };
 
-template <int SIGMA, typename V, typename IT, bool B0>
+template <int SIGMA, typename V, typename IT, bool B0, bool HOT = false>
 __global__ void __launch_bounds__(kT)
 k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restrict__ val,
        const int64_t *__restrict__ tile_ptr, const int64_t *__restrict__ row_lo,
        const unsigned *__restrict__ desc, const int64_t *__restrict__ map_off,
        const int64_t *__restrict__ seg_map, int64_t n_tiles, int64_t nnz,
-       const V *__restrict__ x, V *__restrict__ y, double alpha, double beta,
+       const V *__restrict__ x, const V *__restrict__ xh, V *__restrict__ y, double alpha, double beta,
        int64_t *__restrict__ carry_row, double *__restrict__ carry_val) {
     constexpr int64_t W = 32 * SIGMA;
     constexpr int kQ = kCsr5Win / 32;
@@ -1346,7 +1354,7 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
             r = tile_ptr[n_tiles];
             if ((int64_t)rp[r] < e) {
                 const int64_t end = rp[r + 1];
-                for (int64_t k = e + lane; k < end; k += 32) s += (double)val[k] * (double)ld_x(x + col[k], px);
+                for (int64_t k = e + lane; k < end; k += 32) s += (double)val[k] * (double)ld_x(xp<HOT>(x, xh, col[k]), px);
             } else {
                 r = -1;
             }
@@ -1381,7 +1389,7 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
     const int y_off = (int)((d >> 16) & 0x1FFu);
     double p[SIGMA];
 #pragma unroll
-    for (int s = 0; s < SIGMA; ++s) p[s] = (double)v[s] * (double)ld_x(x + c[s], px);
+    for (int s = 0; s < SIGMA; ++s) p[s] = (double)v[s] * (double)ld_x(xp<HOT>(x, xh, c[s]), px);
     __syncwarp();
 
     auto emit = [&](int idx, double sum) {
@@ -1531,24 +1539,25 @@ spmv_status launch_fixup(spmv_handle *h, V *y, double alpha, cudaStream_t s) {
 
 // ELL rows-per-thread x slot-batch variant; SPMV_ELL_VARIANT="RB" (e.g. 18, 24, 42) overrides the
 // dtype default for tuning experiments (tools/exp.py)
-template <typename V, bool B0>
+template <typename V, bool B0, bool HOT>
 spmv_status launch_ell(spmv_handle *h, const V *x, V *y, double alpha, double beta, cudaStream_t s) {
+    const V *xh = reinterpret_cast<const V *>(h->xhot.p);
     const int64_t n = h->n_rows;
     if (n == 0) return SPMV_OK;
     static const int var = [] { const char *e = getenv("SPMV_ELL_VARIANT"); return e ? atoi(e) : 0; }();
     const int *c = (const int *)h->arr[SPMV_ARR_ELL_COL].p;
     const V *v = (const V *)h->arr[SPMV_ARR_ELL_VAL].p;
     switch (var) {
-    case 14: k_ell<V, B0, 1, 4><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
-    case 28: k_ell<V, B0, 2, 8><<<grid_stride_blocks(h->ctx, (n + 1) / 2, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
-    case 42: k_ell<V, B0, 4, 2><<<grid_stride_blocks(h->ctx, (n + 3) / 4, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
-    case 44: k_ell<V, B0, 4, 4><<<grid_stride_blocks(h->ctx, (n + 3) / 4, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
-    case 18: k_ell<V, B0, 1, 8><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta); break;
+    case 14: k_ell<V, B0, 1, 4, HOT><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, xh, y, n, alpha, beta); break;
+    case 28: k_ell<V, B0, 2, 8, HOT><<<grid_stride_blocks(h->ctx, (n + 1) / 2, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, xh, y, n, alpha, beta); break;
+    case 42: k_ell<V, B0, 4, 2, HOT><<<grid_stride_blocks(h->ctx, (n + 3) / 4, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, xh, y, n, alpha, beta); break;
+    case 44: k_ell<V, B0, 4, 4, HOT><<<grid_stride_blocks(h->ctx, (n + 3) / 4, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, xh, y, n, alpha, beta); break;
+    case 18: k_ell<V, B0, 1, 8, HOT><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, xh, y, n, alpha, beta); break;
     default:   // 16-byte value loads: fp64 2 rows x 4-slot batch, fp32 4 rows x 2-slot batch (measured best)
         if (sizeof(V) == 8)
-            k_ell<V, B0, 2, 4><<<grid_stride_blocks(h->ctx, (n + 1) / 2, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta);
+            k_ell<V, B0, 2, 4, HOT><<<grid_stride_blocks(h->ctx, (n + 1) / 2, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, xh, y, n, alpha, beta);
         else
-            k_ell<V, B0, 4, 2><<<grid_stride_blocks(h->ctx, (n + 3) / 4, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, y, n, alpha, beta);
+            k_ell<V, B0, 4, 2, HOT><<<grid_stride_blocks(h->ctx, (n + 3) / 4, 16), kT, 0, s>>>(c, v, h->ell_K, h->ell_ld, x, xh, y, n, alpha, beta);
         break;
     }
     SPMV_LAUNCH_CHECK();
@@ -1583,20 +1592,21 @@ inline unsigned long long *csr_sched(const spmv_handle *h, int64_t n, int w) {
                                                                                  : nullptr;
 }
 
-template <typename V, typename IT, bool B0>
+template <typename V, typename IT, bool B0, bool HOT>
 spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col, const V *val, const V *x, V *y,
                               int64_t n, int w, double alpha, double beta, cudaStream_t s,
                               int64_t long_len = INT64_MAX, bool pdl = false) {
     if (n == 0) return SPMV_OK;
+    const V *xh = reinterpret_cast<const V *>(h->xhot.p);
     // W <= 8: 32-row batches (A29) when col/val are 32-byte aligned (the chunk loads)
     static const int rows_on = [] { const char *e = getenv("SPMV_CSR_ROWS"); return e ? atoi(e) : 1; }();
     const int wmax = rows_on >= 8 ? rows_on : 8;          // experiment knob: SPMV_CSR_ROWS=16/32 widens it
     if (w <= wmax && rows_on && ((((uintptr_t)col) | ((uintptr_t)val)) & 31) == 0) {
         const unsigned gr = (unsigned)std::min<int64_t>(ceil_div<int64_t>(n, kT), (int64_t)h->ctx->sm_count * kCsrRowsMB);
         if (long_len == INT64_MAX)
-            SPMV_CUDA_TRY(launch_k(k_csr_rows<V, IT, B0, kCsrRowsMB, false>, gr, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len));
+            SPMV_CUDA_TRY(launch_k(k_csr_rows<V, IT, B0, kCsrRowsMB, false, HOT>, gr, s, pdl, rp, col, val, x, xh, y, n, alpha, beta, long_len));
         else
-            SPMV_CUDA_TRY(launch_k(k_csr_rows<V, IT, B0, kCsrRowsMB, true>, gr, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len));
+            SPMV_CUDA_TRY(launch_k(k_csr_rows<V, IT, B0, kCsrRowsMB, true, HOT>, gr, s, pdl, rp, col, val, x, xh, y, n, alpha, beta, long_len));
         return SPMV_OK;
     }
     // 16 CTAs (4096 threads) per SM of grid-stride warps
@@ -1609,13 +1619,13 @@ spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col
     const int gd = sch ? (int)std::min<int64_t>(g, (int64_t)h->ctx->sm_count * 3) : g;
 #define SPMV_VEC(WW)                                                                                           \
     if (sch && long_len == INT64_MAX)                                                                          \
-        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false, true>, gd, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len, sch)); \
+        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false, true, HOT>, gd, s, pdl, rp, col, val, x, xh, y, n, alpha, beta, long_len, sch)); \
     else if (sch)                                                                                              \
-        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true, true>, gd, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len, sch)); \
+        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true, true, HOT>, gd, s, pdl, rp, col, val, x, xh, y, n, alpha, beta, long_len, sch)); \
     else if (long_len == INT64_MAX)                                                                            \
-        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false>, g, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len, nosch)); \
+        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), false, false, HOT>, g, s, pdl, rp, col, val, x, xh, y, n, alpha, beta, long_len, nosch)); \
     else                                                                                                       \
-        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true>, g, s, pdl, rp, col, val, x, y, n, alpha, beta, long_len, nosch))
+        SPMV_CUDA_TRY(launch_k(k_csr_vector<V, IT, WW, B0, (WW <= 8 ? 4 : 3), true, false, HOT>, g, s, pdl, rp, col, val, x, xh, y, n, alpha, beta, long_len, nosch))
     unsigned long long *nosch = nullptr;
     switch (w) {
     case 1: case 2: SPMV_VEC(2); break;
@@ -1629,10 +1639,17 @@ spmv_status launch_csr_vector(const spmv_handle *h, const IT *rp, const int *col
     return SPMV_OK;
 }
 
-template <typename V, typename IT, bool B0>
+template <typename V, typename IT, bool B0, bool HOT>
 spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, cudaStream_t s) {
     if (alpha == 0.0) return launch_scale<V, B0>(h, y, beta, s);   // A14: A not read
     const int64_t n = h->n_rows;
+    // hot columns (A30): this run's x values of the handle's hot set, packed densely
+    const V *xh = reinterpret_cast<const V *>(h->xhot.p);
+    if (h->n_hot > 0) {
+        k_hot_gather<V><<<grid_stride_blocks(h->ctx, h->n_hot, 4), kT, 0, s>>>(
+            x, (const int *)h->arr[SPMV_ARR_HOT_COLS].p, h->n_hot, reinterpret_cast<V *>(h->xhot.p));
+        SPMV_LAUNCH_CHECK();
+    }
     const IT *rp = (const IT *)h->arr[SPMV_ARR_ROW_PTR].p;
     const int *col = (const int *)h->arr[SPMV_ARR_COL].p;
     const V *val = (const V *)h->arr[SPMV_ARR_VAL].p;
@@ -1641,7 +1658,7 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
     switch (h->fmt) {
     case SPMV_CSR:
     {
-        if (h->csr_chunks == 0) return launch_csr_vector<V, IT, B0>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s);
+        if (h->csr_chunks == 0) return launch_csr_vector<V, IT, B0, HOT>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s);
         // long-row chunks first, the row kernel programmatically dependent on them (PDL):
         // the two are independent and run side by side; the chunk grid is one resident
         // wave of chunk_ctas (2) CTAs/SM so that the row kernel's CTAs start at once beside it
@@ -1650,44 +1667,44 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
         if (pdl_on) {
             if (unsigned long long *sch = csr_sched(h, n, (int)h->vec_w)) SPMV_CUDA_TRY(cudaMemsetAsync(sch, 0, 8, s));
         } else {
-            SPMV_TRY((launch_csr_vector<V, IT, B0>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s,
+            SPMV_TRY((launch_csr_vector<V, IT, B0, HOT>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s,
                                                    2 * h->csr_chunk)));
         }
         const int64_t warps = h->csr_chunks;
         const unsigned gc = (unsigned)std::min<int64_t>(ceil_div<int64_t>(warps, kT / 32),
                                                         (int64_t)h->ctx->sm_count * (pdl_on ? chunk_ctas : 16));
-        k_csr_chunks<V, IT><<<gc, kT, 0, s>>>(rp, col, val, (const int64_t *)h->arr[SPMV_ARR_CSR_CHUNK_ROW].p,
+        k_csr_chunks<V, IT, HOT><<<gc, kT, 0, s>>>(rp, col, val, (const int64_t *)h->arr[SPMV_ARR_CSR_CHUNK_ROW].p,
                                               (const int64_t *)h->arr[SPMV_ARR_CSR_CHUNK_LO].p, h->csr_chunks,
-                                              h->csr_chunk, x, crow, cval);
+                                              h->csr_chunk, x, xh, crow, cval);
         SPMV_LAUNCH_CHECK();
         if (pdl_on)
-            SPMV_TRY((launch_csr_vector<V, IT, B0>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s,
+            SPMV_TRY((launch_csr_vector<V, IT, B0, HOT>(h, rp, col, val, x, y, n, (int)h->vec_w, alpha, beta, s,
                                                    2 * h->csr_chunk, true)));
         return launch_fixup<V>(h, y, alpha, s);
     }
     case SPMV_CSR_SCALAR:
         if (n == 0) return SPMV_OK;
-        k_csr_scalar<V, IT, B0><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(rp, col, val, x, y, n, alpha, beta);
+        k_csr_scalar<V, IT, B0, HOT><<<grid_stride_blocks(h->ctx, n, 16), kT, 0, s>>>(rp, col, val, x, xh, y, n, alpha, beta);
         SPMV_LAUNCH_CHECK();
         return SPMV_OK;
     case SPMV_ELL:
         if (n == 0) return SPMV_OK;
-        return launch_ell<V, B0>(h, x, y, alpha, beta, s);
+        return launch_ell<V, B0, HOT>(h, x, y, alpha, beta, s);
     case SPMV_HYB: {
         if (n == 0) return SPMV_OK;
-        SPMV_TRY((launch_ell<V, B0>(h, x, y, alpha, beta, s)));
+        SPMV_TRY((launch_ell<V, B0, HOT>(h, x, y, alpha, beta, s)));
         if (h->hyb_coo_nnz == 0) return SPMV_OK;
-        k_coo<V, true, B0><<<(unsigned)ceil_div<int64_t>(h->n_carry, kT / 32), kT, 0, s>>>(
+        k_coo<V, true, B0, HOT><<<(unsigned)ceil_div<int64_t>(h->n_carry, kT / 32), kT, 0, s>>>(
             (const int *)h->arr[SPMV_ARR_COO_ROW].p, (const int *)h->arr[SPMV_ARR_HYB_COO_COL].p,
-            (const V *)h->arr[SPMV_ARR_HYB_COO_VAL].p, h->hyb_coo_nnz, h->n_carry, x, y, n, alpha, beta, crow, cval);
+            (const V *)h->arr[SPMV_ARR_HYB_COO_VAL].p, h->hyb_coo_nnz, h->n_carry, x, xh, y, n, alpha, beta, crow, cval);
         SPMV_LAUNCH_CHECK();
         return launch_fixup<V>(h, y, alpha, s);
     }
     case SPMV_COO:
         if (h->nnz == 0) return launch_scale<V, B0>(h, y, beta, s);
-        carveout(k_coo<V, false, B0>);
-        k_coo<V, false, B0><<<(unsigned)ceil_div<int64_t>(h->n_carry, kT / 32), kT, 0, s>>>(
-            (const int *)h->arr[SPMV_ARR_COO_ROW].p, col, val, h->nnz, h->n_carry, x, y, n, alpha, beta, crow, cval);
+        carveout(k_coo<V, false, B0, HOT>);
+        k_coo<V, false, B0, HOT><<<(unsigned)ceil_div<int64_t>(h->n_carry, kT / 32), kT, 0, s>>>(
+            (const int *)h->arr[SPMV_ARR_COO_ROW].p, col, val, h->nnz, h->n_carry, x, xh, y, n, alpha, beta, crow, cval);
         SPMV_LAUNCH_CHECK();
         return launch_fixup<V>(h, y, alpha, s);
     case SPMV_MERGE:
@@ -1700,7 +1717,7 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
         // measured 2 % faster than one tile per warp at 4 CTAs/SM (LAP4096, R-MAT 24);
         // T = 128: one tile per warp at 6 CTAs/SM
         if (h->merge_T == 128) {
-            k_merge<V, IT, B0, 4, 6><<<g, kT, 0, s>>>(rp, col, val, cr, h->merge_tiles, dmax, x, y, alpha, beta, crow, cval);
+            k_merge<V, IT, B0, 4, 6, HOT><<<g, kT, 0, s>>>(rp, col, val, cr, h->merge_tiles, dmax, x, xh, y, alpha, beta, crow, cval);
         } else {
             // T = 256 (A28): all tiles class 1 -> the row-sum kernel over all tiles; most
             // (>= half) class 1 -> the row-sum kernel over the class-1 part of the tile order,
@@ -1712,26 +1729,26 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
             const unsigned gr = (unsigned)std::min<int64_t>(ceil_div<int64_t>(nl, kT / 32), (int64_t)h->ctx->sm_count * kMergeRowsMB);
             static const bool pairs = [] { const char *e = getenv("SPMV_MERGE_PAIRS"); return !e || atoi(e) != 0; }();
             if (nl == nt && !pairs) {
-                carveout(k_merge_rows<V, IT, B0, kMergeRowsMB, false, false>);
-                k_merge_rows<V, IT, B0, kMergeRowsMB, false, false><<<gr, kT, 0, s>>>(rp, col, val, cr, ord, 0, nt, dmax, x, y,
+                carveout(k_merge_rows<V, IT, B0, kMergeRowsMB, false, false, HOT>);
+                k_merge_rows<V, IT, B0, kMergeRowsMB, false, false, HOT><<<gr, kT, 0, s>>>(rp, col, val, cr, ord, 0, nt, dmax, x, xh, y,
                                                                                alpha, beta, crow, cval);
             } else if (nl == nt) {
-                carveout(k_merge_rows<V, IT, B0, kMergeRowsMB, false>);
-                k_merge_rows<V, IT, B0, kMergeRowsMB, false><<<gr, kT, 0, s>>>(rp, col, val, cr, ord, 0, nt, dmax, x, y,
+                carveout(k_merge_rows<V, IT, B0, kMergeRowsMB, false, true, HOT>);
+                k_merge_rows<V, IT, B0, kMergeRowsMB, false, true, HOT><<<gr, kT, 0, s>>>(rp, col, val, cr, ord, 0, nt, dmax, x, xh, y,
                                                                                alpha, beta, crow, cval);
             } else if (2 * nl >= nt) {
-                carveout(k_merge_rows<V, IT, B0, kMergeRowsMB, true>);
-                k_merge_rows<V, IT, B0, kMergeRowsMB, true><<<gr, kT, 0, s>>>(rp, col, val, cr, ord, 0, nl, dmax, x, y,
+                carveout(k_merge_rows<V, IT, B0, kMergeRowsMB, true, true, HOT>);
+                k_merge_rows<V, IT, B0, kMergeRowsMB, true, true, HOT><<<gr, kT, 0, s>>>(rp, col, val, cr, ord, 0, nl, dmax, x, xh, y,
                                                                               alpha, beta, crow, cval);
                 SPMV_LAUNCH_CHECK();
                 const unsigned gp = (unsigned)std::min<int64_t>(ceil_div<int64_t>(nt - nl, kT / 32), (int64_t)h->ctx->sm_count * 3);
-                carveout(k_merge_persist<V, IT, B0, 8, 3, true>);
-                k_merge_persist<V, IT, B0, 8, 3, true><<<gp, kT, 0, s>>>(rp, col, val, cr, ord, nl, nt, dmax, x, y, alpha,
+                carveout(k_merge_persist<V, IT, B0, 8, 3, true, HOT>);
+                k_merge_persist<V, IT, B0, 8, 3, true, HOT><<<gp, kT, 0, s>>>(rp, col, val, cr, ord, nl, nt, dmax, x, xh, y, alpha,
                                                                          beta, crow, cval);
             } else {
                 const unsigned gp = (unsigned)std::min<int64_t>(g, (int64_t)h->ctx->sm_count * 3);
-                carveout(k_merge_persist<V, IT, B0, 8, 3, false>);
-                k_merge_persist<V, IT, B0, 8, 3, false><<<gp, kT, 0, s>>>(rp, col, val, cr, ord, 0, nt, dmax, x, y, alpha,
+                carveout(k_merge_persist<V, IT, B0, 8, 3, false, HOT>);
+                k_merge_persist<V, IT, B0, 8, 3, false, HOT><<<gp, kT, 0, s>>>(rp, col, val, cr, ord, 0, nt, dmax, x, xh, y, alpha,
                                                                           beta, crow, cval);
             }
         }
@@ -1742,13 +1759,13 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
         const int64_t warps = h->n_tiles + 1;
         const unsigned g = (unsigned)ceil_div<int64_t>(warps * 32, kT);
 #define SPMV_CSR5_LAUNCH(SG)                                                                                  \
-    carveout(k_csr5<SG, V, IT, B0>);                                                                          \
-    k_csr5<SG, V, IT, B0><<<g, kT, 0, s>>>(rp, col, val, (const int64_t *)h->arr[SPMV_ARR_CSR5_TILE_PTR].p,   \
+    carveout(k_csr5<SG, V, IT, B0, HOT>);                                                                          \
+    k_csr5<SG, V, IT, B0, HOT><<<g, kT, 0, s>>>(rp, col, val, (const int64_t *)h->arr[SPMV_ARR_CSR5_TILE_PTR].p,   \
                                            (const int64_t *)h->arr[SPMV_ARR_CSR5_ROW_LO].p,                    \
                                            (const unsigned *)h->arr[SPMV_ARR_CSR5_TILE_DESC].p,                \
                                            (const int64_t *)h->arr[SPMV_ARR_CSR5_MAP_OFF].p,                   \
                                            (const int64_t *)h->arr[SPMV_ARR_CSR5_SEG_MAP].p, h->n_tiles,       \
-                                           h->nnz, x, y, alpha, beta, crow, cval)
+                                           h->nnz, x, xh, y, alpha, beta, crow, cval)
         switch (h->sigma) {
         case 4: SPMV_CSR5_LAUNCH(4); break;
         case 8: SPMV_CSR5_LAUNCH(8); break;
@@ -1760,7 +1777,7 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
         // rows that start in the tail (< one tile of nonzeros left): CSR-vector
         const int64_t r_tail = h->csr5_tail_row;
         if (r_tail < n)
-            SPMV_TRY((launch_csr_vector<V, IT, B0>(h, rp + r_tail, col, val, x, y + r_tail, n - r_tail, 32, alpha,
+            SPMV_TRY((launch_csr_vector<V, IT, B0, HOT>(h, rp + r_tail, col, val, x, y + r_tail, n - r_tail, 32, alpha,
                                                    beta, s)));
         return launch_fixup<V>(h, y, alpha, s);
     }
@@ -1769,14 +1786,21 @@ spmv_status run_t(spmv_handle *h, double alpha, double beta, const V *x, V *y, c
     return SPMV_ERR_INVALID_ARG;
 }
 
+// beta == 0 (y write-only, A14) and hot columns (A30) are compile-time kernel variants
+template <typename V, typename IT>
+spmv_status run_b(spmv_handle *h, double alpha, double beta, const V *x, V *y, cudaStream_t s) {
+    if (h->n_hot > 0)
+        return beta == 0.0 ? run_t<V, IT, true, true>(h, alpha, beta, x, y, s) : run_t<V, IT, false, true>(h, alpha, beta, x, y, s);
+    return beta == 0.0 ? run_t<V, IT, true, false>(h, alpha, beta, x, y, s) : run_t<V, IT, false, false>(h, alpha, beta, x, y, s);
+}
+
 template <typename V>
 spmv_status run_v(spmv_handle *h, double alpha, double beta, const void *x, void *y, cudaStream_t s) {
     const V *xv = (const V *)x;
     V *yv = (V *)y;
     if (h->itype == SPMV_I32)
-        return beta == 0.0 ? run_t<V, int, true>(h, alpha, beta, xv, yv, s) : run_t<V, int, false>(h, alpha, beta, xv, yv, s);
-    return beta == 0.0 ? run_t<V, int64_t, true>(h, alpha, beta, xv, yv, s)
-                       : run_t<V, int64_t, false>(h, alpha, beta, xv, yv, s);
+        return run_b<V, int>(h, alpha, beta, xv, yv, s);
+    return run_b<V, int64_t>(h, alpha, beta, xv, yv, s);
 }
 
 }  // namespace

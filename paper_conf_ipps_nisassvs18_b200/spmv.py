@@ -29,7 +29,7 @@ ARRAYS = {"row_ptr": 0, "col": 1, "val": 2, "coo_row": 3, "ell_col": 4, "ell_val
           "hyb_coo_val": 7, "merge_coord_row": 8, "merge_coord_nz": 9, "csr5_tile_ptr": 10,
           "csr5_row_lo": 11, "csr5_tile_desc": 12, "csr5_map_off": 13, "csr5_seg_map": 14,
           "csr_chunk_row": 15, "csr_chunk_lo": 16, "merge_tile_class": 17,
-          "merge_tile_order": 18}
+          "merge_tile_order": 18, "hot_cols": 19}
 
 
 class SpmvError(RuntimeError):
@@ -74,7 +74,7 @@ class spmv_convert_opts(C.Structure):
     _fields_ = [("hyb_rule", C.c_int), ("hyb_width", C.c_int64), ("csr5_sigma", C.c_int),
                 ("merge_items", C.c_int), ("vector_width", C.c_int), ("max_bytes", C.c_size_t),
                 ("alias_input", C.c_int), ("index64", C.c_int), ("csr_chunk", C.c_int64),
-                ("features", C.POINTER(spmv_features_t))]
+                ("hot_x", C.c_int64), ("features", C.POINTER(spmv_features_t))]
 
 
 class spmv_handle_info(C.Structure):
@@ -83,7 +83,8 @@ class spmv_handle_info(C.Structure):
                 ("ell_width", C.c_int64), ("ell_ld", C.c_int64), ("hyb_coo_nnz", C.c_int64),
                 ("csr5_sigma", C.c_int64), ("csr5_tiles", C.c_int64), ("csr5_map_len", C.c_int64),
                 ("merge_items", C.c_int64), ("merge_tiles", C.c_int64), ("vector_width", C.c_int64),
-                ("csr_chunks", C.c_int64), ("device_bytes", C.c_size_t), ("bytes_per_run", C.c_size_t),
+                ("csr_chunks", C.c_int64), ("hot_cols", C.c_int64), ("device_bytes", C.c_size_t),
+                ("bytes_per_run", C.c_size_t),
                 ("bytes_per_run_beta0", C.c_size_t)]
 
 
@@ -491,7 +492,7 @@ class Handle:
               "merge_coord_row": np.int64, "merge_coord_nz": np.int64, "csr5_tile_ptr": np.int64,
               "csr5_row_lo": np.int64, "csr5_tile_desc": np.uint32, "csr5_map_off": np.int64,
               "csr5_seg_map": np.int64, "csr_chunk_row": np.int64, "csr_chunk_lo": np.int64,
-              "merge_tile_class": np.uint8, "merge_tile_order": np.int32}[name]
+              "merge_tile_class": np.uint8, "merge_tile_order": np.int32, "hot_cols": np.int32}[name]
         return buf.view(dt)
 
     def destroy(self, stream=None):

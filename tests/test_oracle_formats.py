@@ -542,3 +542,35 @@ def test_oracle_halo_colmap_brute_force(case, P):
             assert np.array_equal(cm[js], snd * S + np.arange(idx.size))
     if case == "lap30" and P > 1:
         assert max(oracle.halo_colmap(A, splits, k)[2] for k in range(P)) <= 30   # one grid line
+
+
+@pytest.mark.parametrize("kmax", [1, 7, 100, 5000, 10 ** 9])
+@pytest.mark.parametrize("case", ["rmat10", "lap30", "ragged", "u2048"])
+def test_oracle_hot_columns_brute_force(case, kmax):
+    """A30: ora_hot_columns == the (kmax+1)-th largest degree rule by sorting; the hot set
+    holds at most kmax columns, every hot column outranks every other referenced column,
+    and the threshold is the smallest that fits."""
+    if case == "rmat10":
+        A = matgen.rmat(10, seed=9)
+    elif case == "lap30":
+        A = matgen.laplacian5(30)
+    elif case == "u2048":
+        A = matgen.uniform_fixed(2048, 2048, 16)
+    else:
+        lens = np.random.default_rng(10).integers(0, 9, 900)
+        lens[600] = 850
+        A = matgen.from_lengths(lens, 900, seed=10)
+    hot = oracle.hot_columns(A, kmax)
+    deg = np.bincount(A.col, minlength=A.n_cols)
+    ref = np.sort(deg)[::-1]
+    if (deg > 0).sum() <= kmax:
+        t = 1
+    else:
+        t = int(ref[kmax]) + 1
+    assert np.array_equal(hot, np.nonzero(deg >= t)[0].astype(np.int32))
+    assert hot.size <= kmax
+    if t > 1:                                   # one lower threshold would exceed the budget
+        assert (deg >= t - 1).sum() > kmax
+    if hot.size:
+        rest = deg[(deg > 0) & (deg < t)]
+        assert rest.size == 0 or rest.max() < deg[hot].min()

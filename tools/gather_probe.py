@@ -59,19 +59,24 @@ def main():
     ap.add_argument("configs", nargs="*", default=["lap4096", "rmat24"])
     ap.add_argument("--reps", type=int, default=50)
     ap.add_argument("--out", default="")
+    ap.add_argument("--formats", default="")
+    ap.add_argument("--modes", default="0,1,2,3")
     a = ap.parse_args()
     lib = build()
     sms = torch.cuda.get_device_properties(0).multi_processor_count
     peak, _ = bench.measured_peak()
     recs = []
     for cfg in a.configs:
-        A = bench.build_matrix(cfg, "f64")
-        dA = sp.CSR.from_host(A)
-        x = torch.from_numpy(matgen.vector(A.n_cols, 1, 1)).cuda()
-        y = torch.from_numpy(matgen.vector(A.n_rows, 1, 2)).cuda()
+        dA, _ = bench.device_matrix(cfg, "f64", torch.float64)     # R-MAT: the GPU generator
+        A = dA
+        from matgen import gpu
+        x = gpu.vector(A.n_cols, 1, 1)
+        y = gpu.vector(A.n_rows, 1, 2)
         out = torch.zeros(1, dtype=torch.float64, device="cuda")
         st = torch.cuda.current_stream().cuda_stream
         for m, what in MODES.items():
+            if str(m) not in a.modes.split(","):
+                continue
             ms = time_fn(lambda: lib.probe_run(m, dA.col.data_ptr(), dA.val.data_ptr(), A.nnz, x.data_ptr(),
                                                out.data_ptr(), sms, st), a.reps)
             byt = 12 * A.nnz
@@ -79,7 +84,7 @@ def main():
                  "stream_gbs": round(byt / ms / 1e6, 1), "gathers_per_ns": round(A.nnz / ms / 1e6, 2)}
             recs.append(r)
             print(json.dumps(r), flush=True)
-        for fmt in sp.PAPER_FORMATS:
+        for fmt in (a.formats.split(",") if a.formats else sp.PAPER_FORMATS):
             try:
                 h = sp.convert(dA, fmt)
             except sp.SpmvError:

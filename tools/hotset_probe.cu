@@ -1,0 +1,74 @@
+// hotset_probe.cu -- experiment: does staging a power-law matrix's hottest x entries in
+// shared memory lift the gather ceiling?  (measurement tool, not the product)
+// Column stream = the matrix's own col/val; cols of the K hottest columns are encoded as
+// -(slot+1) and served from a dense shared copy of x[hot] (persistent CTAs, one per SM).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace {
+__device__ __forceinline__ uint64_t pol_first() { uint64_t p; asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p)); return p; }
+__device__ __forceinline__ uint64_t pol_last() { uint64_t p; asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p)); return p; }
+__device__ __forceinline__ void ld8i(const int *p, int (&v)[8], uint64_t pol) {
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+                 : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]) : "l"(p), "l"(pol));
+}
+__device__ __forceinline__ void ld4d(const double *p, double (&v)[4], uint64_t pol) {
+    long long w[4];
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.b64 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=l"(w[0]), "=l"(w[1]), "=l"(w[2]), "=l"(w[3]) : "l"(p), "l"(pol));
+    for (int i = 0; i < 4; ++i) v[i] = __longlong_as_double(w[i]);
+}
+__device__ __forceinline__ double gx(const double *p, uint64_t pol) {
+    double v; asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(pol)); return v;
+}
+
+template <int HOT>   // 0: all from x; 1: hot from shared memory; 2: hot from a dense global copy
+__global__ void k_hp(const int *__restrict__ col, const double *__restrict__ val, int64_t nnz, const double *__restrict__ x,
+                     const double *__restrict__ xhot, int K, double *__restrict__ out) {
+    extern __shared__ double s_hot[];
+    if (HOT == 1) {
+        for (int i = threadIdx.x; i < K; i += blockDim.x) s_hot[i] = xhot[i];
+        __syncthreads();
+    }
+    const int lane = threadIdx.x & 31;
+    const uint64_t pa = pol_first(), px = pol_last();
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    double s = 0.0;
+    for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * 256 < nnz; w += nw) {
+        const int64_t e0 = w * 256 + lane * 8;
+        int c[8]; double v[8];
+        if (e0 + 8 <= nnz) {
+            ld8i(col + e0, c, pa);
+            double a[4], b[4];
+            ld4d(val + e0, a, pa); ld4d(val + e0 + 4, b, pa);
+            for (int q = 0; q < 4; ++q) { v[q] = a[q]; v[4 + q] = b[q]; }
+        } else {
+            for (int q = 0; q < 8; ++q) { const bool in = e0 + q < nnz; c[q] = in ? col[e0 + q] : 0; v[q] = in ? val[e0 + q] : 0.0; }
+        }
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            double xv;
+            if (HOT == 1 && c[q] < 0) xv = s_hot[-c[q] - 1];
+            else if (HOT == 2 && c[q] < 0) xv = gx(xhot + (-c[q] - 1), px);
+            else xv = gx(x + c[q], px);
+            s += v[q] * xv;
+        }
+    }
+    if (s == 1.2345e300) out[0] = s;
+}
+}  // namespace
+
+extern "C" int hp_run(int hot, const int *col, const double *val, int64_t nnz, const double *x, const double *xhot, int K,
+                      int blocks, int threads, double *out, void *stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    size_t sm = hot == 1 ? (size_t)K * 8 : 0;
+    if (hot == 1) {
+        cudaFuncSetAttribute(k_hp<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        k_hp<1><<<blocks, threads, sm, s>>>(col, val, nnz, x, xhot, K, out);
+    } else if (hot == 2) {
+        k_hp<2><<<blocks, threads, 0, s>>>(col, val, nnz, x, xhot, K, out);
+    } else {
+        k_hp<0><<<blocks, threads, 0, s>>>(col, val, nnz, x, xhot, K, out);
+    }
+    return (int)cudaGetLastError();
+}
