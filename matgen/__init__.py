@@ -215,22 +215,40 @@ def _loguniform(rng, lo, hi):
     return float(np.exp(rng.uniform(np.log(lo), np.log(hi))))
 
 
+def nnz_bucket(nnz):
+    """Index of the Table I bucket holding nnz (-1: outside all)."""
+    for k, (lo, hi, _) in enumerate(NNZ_BUCKETS):
+        if lo <= nnz < hi or (k == len(NNZ_BUCKETS) - 1 and nnz == hi):
+            return k
+    return -1
+
+
 def sweep_params(i, max_nnz=None):
     """Parameters of sweep matrix i: family = i mod 5,
-    nnz bucket drawn with Table I frequencies, log-uniform within it; mu log-uniform in
-    [1, 256]; n_rows = max(8, nnz/mu); 80% square, else aspect log-uniform in [1/4, 4]."""
+    nnz bucket drawn with Table I frequencies, log-uniform within it (cap 96M, PAPER.md:117);
+    mu log-uniform in [1, 256]; n_rows = max(8, nnz/mu); 80% square, else aspect
+    log-uniform in [1/4, 4]; the shape is widened where n_rows x n_cols could not hold
+    1.25 x the target (tiny matrices with long rows)."""
     rng = np.random.default_rng(SEEDS["sweep"] + i)
     fam = FAMILIES[i % 5]
     w = np.array([b[2] for b in NNZ_BUCKETS], dtype=float)
-    b = NNZ_BUCKETS[int(rng.choice(len(NNZ_BUCKETS), p=w / w.sum()))]
+    bk = int(rng.choice(len(NNZ_BUCKETS), p=w / w.sum()))
+    b = NNZ_BUCKETS[bk]
     nnz = int(_loguniform(rng, b[0], b[1]))
     if max_nnz:
         nnz = min(nnz, int(max_nnz))
     mu = _loguniform(rng, 1.0, 256.0)
     n_rows = max(8, int(nnz / mu))
-    aspect = 1.0 if rng.random() < 0.8 else _loguniform(rng, 0.25, 4.0)
+    square = rng.random() < 0.8
+    aspect = 1.0 if square else _loguniform(rng, 0.25, 4.0)
     n_cols = max(8, int(n_rows * aspect))
-    p = dict(i=i, family=fam, nnz_target=nnz, mu=mu, n_rows=n_rows, n_cols=n_cols, seed=SEEDS["sweep"] + i)
+    if n_rows * n_cols < 1.25 * nnz:
+        if square:
+            n_rows = n_cols = int(np.ceil(np.sqrt(1.25 * nnz)))
+        else:
+            n_cols = int(np.ceil(1.25 * nnz / n_rows))
+    p = dict(i=i, family=fam, nnz_target=nnz, bucket=bk, mu=mu, n_rows=n_rows, n_cols=n_cols,
+             seed=SEEDS["sweep"] + i)
     if fam == "banded":
         p["fill"] = float(rng.uniform(0.3, 1.0))
     elif fam == "blockdiag":
@@ -248,6 +266,34 @@ def sweep_params(i, max_nnz=None):
     return p
 
 
+def fit_lengths(lens, target, m):
+    """Row lengths rescaled to sum exactly to `target` with each <= m (water-filling over
+    the rows below the cap, then largest-remainder rounding): the family's length
+    distribution kept, its total pinned to the nnz target."""
+    lens = np.asarray(lens, dtype=np.float64)
+    n = lens.size
+    target = int(min(target, n * m))
+    if n == 0 or target == 0:
+        return np.zeros(n, dtype=np.int64)
+    s = lens if lens.sum() > 0 else np.ones(n)
+    s = s / s.sum() * target
+    for _ in range(64):
+        s = np.minimum(s, m)
+        short = target - s.sum()
+        free = s < m
+        if short <= 1e-9 or not free.any():
+            break
+        base = s[free].sum()
+        s[free] = s[free] * (1.0 + short / base) if base > 0 else s[free] + short / free.sum()
+    s = np.minimum(s, m)
+    out = np.floor(s).astype(np.int64)
+    rem = int(target - out.sum())
+    if rem > 0:
+        frac = np.where(out < m, s - out, -1.0)
+        out[np.argsort(-frac, kind="stable")[:rem]] += 1
+    return np.minimum(out, m)
+
+
 def _union_rows(A: HostCSR, B: HostCSR) -> HostCSR:
     """Row-wise union of two structures (duplicates coalesced; A's values kept)."""
     ra = np.repeat(np.arange(A.n_rows, dtype=np.int64), np.diff(A.row_ptr))
@@ -262,31 +308,44 @@ def _union_rows(A: HostCSR, B: HostCSR) -> HostCSR:
 
 
 def sweep_matrix(i, kind="f64", max_nnz=None):
-    """Build sweep matrix i (canonical CSR, seeded values).  Returns (HostCSR, params)."""
+    """Build sweep matrix i (canonical CSR, seeded values).  Returns (HostCSR, params).
+    Length-drawn families (uniform, power-law, mixed) have their row lengths pinned to
+    the nnz target (fit_lengths); window families (banded, block-diagonal) are resized
+    (rows scaled by target / realized, up to 4 tries) until the realized nnz falls in the
+    target's Table I bucket.  params["nnz"] records the realized count."""
     p = sweep_params(i, max_nnz)
-    rng = np.random.default_rng(p["seed"] + 1)
     n, m, mu, seed = p["n_rows"], p["n_cols"], p["mu"], p["seed"]
     fam = p["family"]
-    if fam == "uniform":
-        lens = np.minimum(rng.poisson(mu, n), m)
-        A = from_lengths(lens, m, seed, kind)
-    elif fam == "banded":
-        half = max(0, int(round(mu / (2 * p["fill"]) - 0.5)))
-        A = window(n, m, half, p["fill"], seed, 0, kind)
-    elif fam == "blockdiag":
-        bsz = min(p["block"], n)
-        base = window(n, m, bsz, p["fill"], seed, 1, "ones")
-        nl = np.minimum(rng.poisson(p["noise"] * max(1.0, base.nnz / n), n), m)
-        noise = from_lengths(nl, m, seed + 3, "ones")
-        A = set_values(_union_rows(base, noise), seed + 5, kind)
-    elif fam == "powerlaw":
-        raw = rng.pareto(p["gamma"] - 1.0, n) + 1.0
-        lens = np.minimum(np.maximum(0, np.round(raw * mu / raw.mean())), m).astype(np.int64)
-        A = from_lengths(lens, m, seed, kind)
-    else:  # mixed
-        lens = rng.poisson(mu, n)
-        long = rng.random(n) < p["q"]
-        lens[long] = (mu * rng.uniform(10.0, p["long"], long.sum())).astype(np.int64)
-        A = from_lengths(np.minimum(lens, m), m, seed, kind)
+    target = p["nnz_target"]
+    if fam in ("uniform", "powerlaw", "mixed"):
+        rng = np.random.default_rng(p["seed"] + 1)
+        if fam == "uniform":
+            lens = rng.poisson(mu, n)
+        elif fam == "powerlaw":
+            lens = rng.pareto(p["gamma"] - 1.0, n) + 1.0
+        else:  # mixed: a fraction q of long rows at 10..long x mu
+            lens = rng.poisson(mu, n).astype(np.float64)
+            long = rng.random(n) < p["q"]
+            lens[long] = mu * rng.uniform(10.0, p["long"], long.sum())
+        A = from_lengths(fit_lengths(lens, target, m), m, seed, kind)
+    else:
+        for _ in range(4):
+            rng = np.random.default_rng(p["seed"] + 1)
+            if fam == "banded":
+                half = max(0, int(round(mu / (2 * p["fill"]) - 0.5)))
+                A = window(n, m, half, p["fill"], seed, 0, kind)
+            else:
+                bsz = min(p["block"], n)
+                base = window(n, m, bsz, p["fill"], seed, 1, "ones")
+                nl = np.minimum(rng.poisson(p["noise"] * max(1.0, base.nnz / n), n), m)
+                noise = from_lengths(nl, m, seed + 3, "ones")
+                A = set_values(_union_rows(base, noise), seed + 5, kind)
+            if nnz_bucket(A.nnz) == nnz_bucket(target) or A.nnz == 0:
+                break
+            f = target / max(A.nnz, 1)
+            n = max(8, int(round(n * f)))
+            m = max(8, int(round(m * f)))
+        p["n_rows"], p["n_cols"] = n, m
+    p["nnz"] = A.nnz
     A.name = f"sweep{i}-{fam}"
     return A, p

@@ -193,9 +193,8 @@ int ora_csr2hyb(int64_t n_rows, const int64_t *row_ptr, const int32_t *col,
     return 0;
 }
 
-/* Merge-based CSR (PAPER.md:103): "logically partitions the work ... into equal
- * sized sub-problems".  Work items = n_rows row ends + nnz nonzeros; tile t takes
- * diagonals [t*T, (t+1)*T). */
+/* CSR long-row chunks (A25): rows longer than 2*C nonzeros are cut into C-nonzero chunks,
+ * listed by row, then chunk index; chunk j of row r starts at row_ptr[r] + j*C. */
 int64_t ora_csr_chunks(int64_t n_rows, const int64_t *row_ptr, int64_t C,
                        int64_t *chunk_row, int64_t *chunk_lo)
 {
@@ -213,6 +212,9 @@ int64_t ora_csr_chunks(int64_t n_rows, const int64_t *row_ptr, int64_t C,
     return k;
 }
 
+/* Merge-based CSR (PAPER.md:103): "logically partitions the work ... into equal
+ * sized sub-problems".  Work items = n_rows row ends + nnz nonzeros; tile t takes
+ * diagonals [t*T, (t+1)*T). */
 int64_t ora_merge_ntiles(int64_t n_rows, int64_t nnz, int64_t T)
 {
     if (T <= 0) return -1;

@@ -31,6 +31,9 @@ LABEL_SETS = {
     "label7": ("coo", "ell", "csr", "hyb", "merge", "csr5", "csr_scalar"),
 }
 LABEL_ORDER = PAPER_FORMATS + ("csr_scalar",)   # exact ties: Fig. 3 order, then the variant
+# largest accepted |y_f - y_csr| / (max |y_csr| + 1) per dtype: 64 x the north_star bound's
+# tolerance (the bound is per row and relative to sum |a||x|; this is a coarse screen)
+AGREE_TOL = {torch.float64: 64 * 1e-12, torch.float32: 64 * 1e-5}
 
 
 class L2Flush:
@@ -154,6 +157,11 @@ def measure_matrix(A: CSR, formats: Iterable[str] = PAPER_FORMATS, reps: int = 5
     rec.update(labels(times))
     if flush is not None:
         rec["cold_labels"] = labels(cold)
+    # a record whose formats disagree beyond the tolerance is not a label
+    tol = AGREE_TOL.get(A.dtype, 1e-5)
+    bad = {f: r["agree"] for f, r in rec["formats"].items() if r.get("agree") is not None and r["agree"] > tol}
+    if bad:
+        rec["rejected"] = {"reason": f"formats disagree with CSR beyond {tol:g} (relative)", "agree": bad}
     return rec
 
 
@@ -202,20 +210,15 @@ def sweep(start: int = 0, count: int = 2000, out: str = "sweep.jsonl", dtype: st
                                                       "n_empty_rows")},
                    "gpu": torch.cuda.get_device_name(), "wall_s": None, **rec}
             row["wall_s"] = round(time.time() - t0, 3)
+            if "rejected" in row:                  # kept aside, never a label
+                with open(out.replace(".jsonl", ".rejected.jsonl"), "a") as rj:
+                    rj.write(json.dumps(row) + "\n")
+                continue
             fh.write(json.dumps(row) + "\n")
             fh.flush()
             n += 1
             del dA
     return n
-
-
-def best_format(rec: Dict[str, object]) -> Optional[str]:
-    return rec.get("label6")  # type: ignore[return-value]
-
-
-def records_to_rows(recs: List[Dict[str, object]]) -> List[Dict[str, object]]:
-    """Flatten measure_matrix records (one JSONL line per matrix)."""
-    return [dict(r) for r in recs]
 
 
 def _main():
@@ -230,13 +233,20 @@ def _main():
     ap.add_argument("--max-nnz", type=int, default=None)
     ap.add_argument("--cold-l2", action="store_true", help="also time every format with L2 flushed before each run")
     ap.add_argument("--with-scalar", action="store_true", help="time CSR-scalar too and emit label7")
+    ap.add_argument("--stride", type=int, default=1, help="only matrices i with i %% stride == 0 (subsets)")
     a = ap.parse_args()
     import os
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
     out = a.out if ws == 1 else a.out.replace(".jsonl", f".rank{rank}.jsonl")
-    n = sweep(a.start, a.count, out, a.dtype, a.reps, a.warmup, rank, ws, a.max_nnz, a.cold_l2, a.with_scalar)
+    if a.stride > 1:                                # i % stride == 0, replicas over i // stride
+        n = 0
+        for i in range(a.start, a.start + a.count):
+            if i % a.stride == 0 and (i // a.stride) % ws == rank:
+                n += sweep(i, 1, out, a.dtype, a.reps, a.warmup, 0, 1, a.max_nnz, a.cold_l2, a.with_scalar)
+    else:
+        n = sweep(a.start, a.count, out, a.dtype, a.reps, a.warmup, rank, ws, a.max_nnz, a.cold_l2, a.with_scalar)
     print(f"rank {rank}: measured {n} matrices -> {out}")
 
 

@@ -50,3 +50,31 @@ def test_sweep_bucket_frequencies():
     expect = np.array([b[2] for b in matgen.NNZ_BUCKETS], float)
     expect = expect / expect.sum() * 2000
     assert np.all(np.abs(counts - expect) < 5 * np.sqrt(expect) + 5)
+
+
+def test_sweep_realized_nnz_in_bucket():
+    """configs[3] fidelity: the REALIZED nnz of every family lands in its target's Table I
+    bucket (cap 96M) -- checked on every third matrix
+    whose target is below 400K nonzeros (the CPU-cheap part of the sweep)."""
+    seen = set()
+    for i in range(0, 2000, 3):
+        p = matgen.sweep_params(i)
+        if p["nnz_target"] > 400_000:
+            continue
+        A, q = matgen.sweep_matrix(i)
+        seen.add(q["family"])
+        assert q["nnz"] == A.nnz
+        assert matgen.nnz_bucket(A.nnz) == q["bucket"], (i, q["family"], q["nnz_target"], A.nnz)
+    assert seen == set(matgen.FAMILIES)
+    assert max(matgen.sweep_params(i)["nnz_target"] for i in range(2000)) <= 96_000_000
+
+
+def test_fit_lengths():
+    """Row lengths pinned to the target sum with the cap respected and the shape kept."""
+    rng = np.random.default_rng(4)
+    lens = rng.pareto(0.8, 5000) + 1.0
+    out = matgen.fit_lengths(lens, 123_457, 300)
+    assert out.sum() == 123_457 and out.max() <= 300 and out.min() >= 0
+    o = out[np.argsort(lens, kind="stable")]
+    assert np.all(np.diff(o) >= -1)                  # order of the drawn lengths kept (up to rounding)
+    assert matgen.fit_lengths(np.ones(10), 1000, 7).sum() == 70           # capped by n x m

@@ -1,7 +1,8 @@
 """Small workload that launches every libspmv kernel, for
 compute-sanitizer: features, all converters, every format's SpMV in fp64/fp32 with
 beta = 0 (NaN y) and beta != 0, alpha = 0, the int64 index path, the CSR long-row
-chunks, partition / slice remap / colmap / gather / own-foreign split.
+chunks, A30 hot columns in every format, the GPU R-MAT generator, partition / slice
+remap / colmap / halo colmap / gather / own-foreign split.
 
 usage: compute-sanitizer --tool memcheck python tools/sanitize_workload.py
 """
@@ -56,6 +57,26 @@ def main():
                         n_launch += h.launches()
                     h.destroy()
         torch.cuda.synchronize()
+    # A30 hot columns forced on every format (the per-run pack + the HOT kernel variants)
+    A = matgen.rmat(13, seed=13)
+    dA = sp.CSR.from_host(A)
+    x = torch.from_numpy(matgen.vector(A.n_cols, 6, 1)).cuda()
+    for fmt in ("coo", "ell", "csr", "hyb", "merge", "csr5"):
+        try:
+            h = sp.convert(dA, fmt, hot_x=64)
+        except sp.SpmvError:
+            continue
+        for beta in (0.0, 1.0):
+            y = torch.zeros(A.n_rows, dtype=torch.float64, device="cuda")
+            h.run(1.0, x, beta, y)
+            n_launch += h.launches()
+        h.export("col") if fmt not in ("ell", "hyb") else h.export("ell_col")
+        h.destroy()
+    # the GPU R-MAT generator (input generation: keys, sort/unique, CSR, values, vectors)
+    from matgen import gpu
+    gpu.rmat(12, seed=14)
+    gpu.vector(1000, 1, 1)
+    torch.cuda.synchronize()
     # CSR-vector with the dynamic batch scheduler (W >= 16, >= 1.8M rows): R-MAT scale 21
     A = matgen.rmat(21, seed=21)
     dA = sp.CSR.from_host(A)
