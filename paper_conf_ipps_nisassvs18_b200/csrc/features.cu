@@ -215,6 +215,9 @@ k_features(const IT *__restrict__ rp, const int *__restrict__ col, int64_t n, in
     // per-lane accumulators
     unsigned long long len2 = 0, over = 0, nb2 = 0, sz2 = 0;
     unsigned len_mn = UINT_MAX, len_mx = 0, n_empty = 0, nb_mn = UINT_MAX, nb_mx = 0, sz_mn = UINT_MAX, sz_mx = 0;
+    // P-typed (32-bit for int32 row_ptr) copies of the bounds the row pass compares with
+    const P nnzP = (P)nnz, khP = (P)(kh < nnz ? kh : nnz);
+    const P hbinP = (P)(hist_bins - 1 < nnz ? (hist_bins - 1 > 0 ? hist_bins - 1 : 0) : nnz);
     // warp-uniform state
     P c_lastflag = kNone;           // position of the last block start so far (kNone: none)
     unsigned c_F = 0;               // block starts so far in the warp's range
@@ -274,17 +277,17 @@ k_features(const IT *__restrict__ rp, const int *__restrict__ col, int64_t n, in
                 P len = bb - a[u];
                 if (inr) {
                     if (arel >= (P)kc_rel && arel < (P)kCap) atomicOr(&bm[(int)arel >> 5], 1u << ((int)arel & 31));
-                    if (len < 0 || a[u] < 0 || (int64_t)bb > nnz) { bad |= BAD_ROWPTR_ORDER; len = 0; }
+                    if (len < 0 || a[u] < 0 || bb > nnzP) { bad |= BAD_ROWPTR_ORDER; len = 0; }
                     const unsigned ul = (unsigned)len;
                     len2 += (unsigned long long)ul * ul;
                     len_mn = min(len_mn, ul);
                     len_mx = max(len_mx, ul);
                     n_empty += len == 0;
-                    over += (int64_t)len > kh ? (unsigned long long)((int64_t)len - kh) : 0ull;
+                    over += (unsigned)(len > khP ? len - khP : (P)0);
                 }
                 if (use_hist) {                                      // empty rows: n_empty (bin 0)
                     const bool hb = inr && len > 0;
-                    const unsigned bin = hb ? (unsigned)((int64_t)len < hist_bins - 1 ? (int64_t)len : hist_bins - 1) : 0u;
+                    const unsigned bin = hb ? (unsigned)(len < hbinP ? len : hbinP) : 0u;
                     const unsigned hm = __ballot_sync(0xffffffffu, hb);
                     if (hm) {
                         const int lead = __ffs(hm) - 1;
@@ -466,28 +469,31 @@ k_features(const IT *__restrict__ rp, const int *__restrict__ col, int64_t n, in
                 const unsigned exo = __shfl_sync(0xffffffffu, ex, o);
                 long long F_first = -1, F_last = -1;
                 if (s1 > s0) {
+                    unsigned Fl = 0;                                  // F of the previous row start
+                    bool have = false;
                     // the (s0 - ex_o)-th row start inside lane o's words
                     unsigned skip = s0 - exo;
                     int wi = o * per;
                     unsigned m = bm[wi] & vmask(wi);
                     while (__popc(m) <= skip) { skip -= __popc(m); ++wi; m = bm[wi] & vmask(wi); }
                     for (; skip; --skip) m &= m - 1u;
+                    F_first = (long long)(F_sub + pf[wi] + __popc(fl[wi] & ((1u << (__ffs(m) - 1)) - 1u)));
                     for (unsigned k = s0; k < s1; ++k) {
                         const int b = __ffs(m) - 1;
-                        const long long Fp = (long long)(F_sub + pf[wi] + __popc(fl[wi] & ((1u << b) - 1u)));
-                        if (F_last >= 0) {
-                            const unsigned nb = (unsigned)(Fp - F_last);
+                        const unsigned Fp = F_sub + pf[wi] + __popc(fl[wi] & ((1u << b) - 1u));
+                        const unsigned nb = Fp - Fl;                  // the previous row's block count
+                        if (have) {
                             nb2 += (unsigned long long)nb * nb;
                             nb_mn = min(nb_mn, nb);
                             nb_mx = max(nb_mx, nb);
-                        } else {
-                            F_first = Fp;
                         }
-                        F_last = Fp;
+                        have = true;
+                        Fl = Fp;
                         m &= m - 1u;
                         if (k + 1 < s1)
                             while (!m) { ++wi; m = bm[wi] & vmask(wi); }
                     }
+                    F_last = (long long)Fl;
                 }
                 // the last row of a lane ends at the next working lane's first row start
                 const unsigned workm = __ballot_sync(0xffffffffu, s1 > s0);

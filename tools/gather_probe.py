@@ -85,6 +85,8 @@ def main():
             recs.append(r)
             print(json.dumps(r), flush=True)
         for fmt in (a.formats.split(",") if a.formats else sp.PAPER_FORMATS):
+            if fmt not in sp.FORMATS:
+                continue
             try:
                 h = sp.convert(dA, fmt)
             except sp.SpmvError:

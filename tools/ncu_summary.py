@@ -152,7 +152,7 @@ def full(rep, out, traffic=None, formats=("coo", "ell", "csr", "hyb", "merge", "
     print("\n".join(lines))
     if traffic:
         cfg, dt = traffic
-        p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+        p = os.environ.get("NCU_TRAFFIC_JSON", os.path.join(ROOT, "profiles", "ncu_traffic.json"))
         d = json.load(open(p)) if os.path.exists(p) else {}
         d.setdefault(cfg, {})[dt] = {k: int(v) for k, v in trafficmap.items()}
         d["_note"] = ("DRAM bytes (read+write) of one spmv_run of each format -- every kernel of the run, "
