@@ -155,6 +155,15 @@ __device__ __forceinline__ const V *xp(const V *x, const V *xh, int c) {
     else return x + c;
 }
 
+
+// x gather of column c (HOT, A30: from the packed hot entries when c <= -2).  Marking the
+// cold gathers evict_first instead of evict_last was measured slower on R-MAT 27 (CSR5
+// 14.1 -> 14.3 ms, merge 21.2 -> 22.0), so both keep the evict_last policy of x.
+template <bool HOT, typename V>
+__device__ __forceinline__ V ldx(const V *x, const V *xh, int c, uint64_t px) {
+    return ld_x(xp<HOT>(x, xh, c), px);
+}
+
 // plain read-only loads for metadata (row_ptr, descriptors)
 template <typename T> __device__ __forceinline__ T ldg(const T *p) { return __ldg(p); }
 

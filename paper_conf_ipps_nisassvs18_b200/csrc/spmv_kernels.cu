@@ -166,7 +166,7 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
         }
         double s[U];
 #pragma unroll
-        for (int u = 0; u < U; ++u) s[u] = c0[u] != -1 ? (double)v0[u] * (double)ld_x(xp<HOT>(x, xh, c0[u]), px) : 0.0;
+        for (int u = 0; u < U; ++u) s[u] = c0[u] != -1 ? (double)v0[u] * (double)ldx<HOT>(x, xh, c0[u], px) : 0.0;
         // the group's U results: lane sub == u of group g writes row u*G + g
         double mine = 0.0;
         {
@@ -229,7 +229,7 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
                         w[q] = in ? ld_hint(val + k + q * SW, pa) : (V)0;
                     }
 #pragma unroll
-                    for (int q = 0; q < 8; ++q) if (d[q] != -1) acc[q] += (double)w[q] * (double)ld_x(xp<HOT>(x, xh, d[q]), px);
+                    for (int q = 0; q < 8; ++q) if (d[q] != -1) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
                 }
                 double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
                 for (int o = SW >> 1; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
@@ -255,14 +255,14 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
 #pragma unroll
                     for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
 #pragma unroll
-                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(xp<HOT>(x, xh, d[q]), px);
+                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
                     if (++it == kFold) {                 // blocked summation (A13)
 #pragma unroll
                         for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
                         it = 0;
                     }
                 }
-                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(xp<HOT>(x, xh, ld_hint(col + k, pa)), px);
+                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ldx<HOT>(x, xh, ld_hint(col + k, pa), px);
                 double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
                 part = warp_sum(tot + part);
                 const int writer = (i / U) * W + i % U;   // lane holding row i's group sum
@@ -310,14 +310,14 @@ k_csr_chunks(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
 #pragma unroll
             for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
 #pragma unroll
-            for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(xp<HOT>(x, xh, d[q]), px);
+            for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
             if (++it == kFold) {
 #pragma unroll
                 for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
                 it = 0;
             }
         }
-        for (; k < hi; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(xp<HOT>(x, xh, ld_hint(col + k, pa)), px);
+        for (; k < hi; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ldx<HOT>(x, xh, ld_hint(col + k, pa), px);
         const double part = warp_sum(tot + (((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]))));
         if (lane == 0) { carry_row[c] = r; carry_val[c] = part; }
     }
@@ -335,10 +335,10 @@ k_csr_scalar(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
         double a0 = 0.0, a1 = 0.0;
         int64_t k = __ldg(rp + r), b = __ldg(rp + r + 1);
         for (; k + 1 < b; k += 2) {
-            a0 += (double)__ldg(val + k) * (double)ld_x(xp<HOT>(x, xh, __ldg(col + k)), px);
-            a1 += (double)__ldg(val + k + 1) * (double)ld_x(xp<HOT>(x, xh, __ldg(col + k + 1)), px);
+            a0 += (double)__ldg(val + k) * (double)ldx<HOT>(x, xh, __ldg(col + k), px);
+            a1 += (double)__ldg(val + k + 1) * (double)ldx<HOT>(x, xh, __ldg(col + k + 1), px);
         }
-        if (k < b) a0 += (double)__ldg(val + k) * (double)ld_x(xp<HOT>(x, xh, __ldg(col + k)), px);
+        if (k < b) a0 += (double)__ldg(val + k) * (double)ldx<HOT>(x, xh, __ldg(col + k), px);
         double o = alpha * (a0 + a1);
         if (!B0) o = fma(beta, yv, o);
         y[r] = (V)o;
@@ -420,10 +420,10 @@ k_ell(const int *__restrict__ ecol, const V *__restrict__ eval, int64_t K, int64
 #pragma unroll
                 for (int u = 0; u < BATCH; u += 2) {
                     const int cu = lane_of(c[u], q);
-                    if (j0 + u < K && cu != -1) a0 += (double)lane_of(v[u], q) * (double)ld_x(xp<HOT>(x, xh, cu), px);
+                    if (j0 + u < K && cu != -1) a0 += (double)lane_of(v[u], q) * (double)ldx<HOT>(x, xh, cu, px);
                     if (u + 1 < BATCH) {
                         const int cw = lane_of(c[u + 1], q);
-                        if (j0 + u + 1 < K && cw != -1) a1 += (double)lane_of(v[u + 1], q) * (double)ld_x(xp<HOT>(x, xh, cw), px);
+                        if (j0 + u + 1 < K && cw != -1) a1 += (double)lane_of(v[u + 1], q) * (double)ldx<HOT>(x, xh, cw, px);
                     }
                 }
                 part[q] += a0 + a1;
@@ -548,7 +548,7 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
     double p[8];
     if constexpr (sizeof(V) == 4) {
 #pragma unroll
-        for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(xp<HOT>(x, xh, c[s]), px) : 0.0;
+        for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ldx<HOT>(x, xh, c[s], px) : 0.0;
     }
     // rows around the tile (uniform loads)
     const int rf = __shfl_sync(0xffffffffu, r[0], 0);                       // tile's first row
@@ -576,7 +576,7 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
     }
     if constexpr (sizeof(V) == 8) {
 #pragma unroll
-        for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ld_x(xp<HOT>(x, xh, c[s]), px) : 0.0;
+        for (int s = 0; s < 8; ++s) p[s] = s < nv ? (double)v[s] * (double)ldx<HOT>(x, xh, c[s], px) : 0.0;
     }
     // rows past the window (sparse stretches: R-MAT's empty rows): the warp first writes
     // beta*y to all of them, 128 rows per step, coalesced; the tile's segments there then
@@ -670,7 +670,7 @@ __device__ __forceinline__ double row_walk(const int *s_c, const V *s_v, int st,
         }
         double pp[8];
 #pragma unroll
-        for (int u = 0; u < 8; ++u) pp[u] = k + u < len ? (double)vv[u] * (double)ld_x(xp<HOT>(x, xh, cc[u]), px) : 0.0;
+        for (int u = 0; u < 8; ++u) pp[u] = k + u < len ? (double)vv[u] * (double)ldx<HOT>(x, xh, cc[u], px) : 0.0;
 #pragma unroll
         for (int u = 0; u < 8; u += 2) { a0 += pp[u]; a1 += pp[u + 1]; }
     }
@@ -693,7 +693,7 @@ __device__ __forceinline__ double row_walk_global(const int *__restrict__ col, c
         }
         double pp[8];
 #pragma unroll
-        for (int u = 0; u < 8; ++u) pp[u] = k + u < len ? (double)vv[u] * (double)ld_x(xp<HOT>(x, xh, cc[u]), px) : 0.0;
+        for (int u = 0; u < 8; ++u) pp[u] = k + u < len ? (double)vv[u] * (double)ldx<HOT>(x, xh, cc[u], px) : 0.0;
 #pragma unroll
         for (int u = 0; u < 8; u += 2) { a0 += pp[u]; a1 += pp[u + 1]; }
     }
@@ -819,14 +819,14 @@ k_csr_rows(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
 #pragma unroll
                     for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
 #pragma unroll
-                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ld_x(xp<HOT>(x, xh, d[q]), px);
+                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
                     if (++it == kFold) {
 #pragma unroll
                         for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
                         it = 0;
                     }
                 }
-                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ld_x(xp<HOT>(x, xh, ld_hint(col + k, pa)), px);
+                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ldx<HOT>(x, xh, ld_hint(col + k, pa), px);
                 const double part = warp_sum(tot + (((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]))));
                 if (lane == i) sum = part;
             }
@@ -939,7 +939,7 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
     double p[LI];
 #pragma unroll
     for (int e = 0; e < LI; ++e)
-        p[e] = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)v[e] * (double)ld_x(xp<HOT>(x, xh, c[e]), px) : 0.0;
+        p[e] = (any && (unsigned)(j0 + e) < (unsigned)nnzt) ? (double)v[e] * (double)ldx<HOT>(x, xh, c[e], px) : 0.0;
     __syncwarp();
     // segment starts: local row i (1 <= i <= nrows) starts at s_end[i-1]; row 0 at 0 if
     // r0_inside.  The bitmap is indexed by chunk position (tile position + off).
@@ -992,7 +992,7 @@ merge_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V *__re
                     cur = pos;
                     acc = 0.0;
                 }
-                acc += (double)ld_hint(val + k0 + pos, pa) * (double)ld_x(xp<HOT>(x, xh, ld_hint(col + k0 + pos, pa)), px);
+                acc += (double)ld_hint(val + k0 + pos, pa) * (double)ldx<HOT>(x, xh, ld_hint(col + k0 + pos, pa), px);
             }
         }
     }
@@ -1216,14 +1216,14 @@ merge_rows_tile(const IT *__restrict__ rp, const int *__restrict__ col, const V 
 #pragma unroll
     for (int e = 0; e < LI; e += 2) {
         const int pe = chunk_pos<V, PAIRS>(lane, e);      // chunk position of element e (pe + 1 of e + 1)
-        const double p0 = (ends_in && (unsigned)(pe - off) < (unsigned)nnzt) ? (double)ch.v[e] * (double)ld_x(xp<HOT>(x, xh, ch.c[e]), px) : 0.0;
-        const double p1 = (ends_in && (unsigned)(pe + 1 - off) < (unsigned)nnzt) ? (double)ch.v[e + 1] * (double)ld_x(xp<HOT>(x, xh, ch.c[e + 1]), px) : 0.0;
+        const double p0 = (ends_in && (unsigned)(pe - off) < (unsigned)nnzt) ? (double)ch.v[e] * (double)ldx<HOT>(x, xh, ch.c[e], px) : 0.0;
+        const double p1 = (ends_in && (unsigned)(pe + 1 - off) < (unsigned)nnzt) ? (double)ch.v[e + 1] * (double)ldx<HOT>(x, xh, ch.c[e + 1], px) : 0.0;
         *reinterpret_cast<double2 *>(s_p + pe) = make_double2(p0, p1);
     }
     if (lane == 31) {                                     // positions past lane 31's chunk (< off row ends)
 #pragma unroll 1
         for (int pos = j0 + LI; pos < nnzt; ++pos)
-            s_p[pos + off] = (double)ld_hint(val + k0 + pos, pa) * (double)ld_x(xp<HOT>(x, xh, ld_hint(col + k0 + pos, pa)), px);
+            s_p[pos + off] = (double)ld_hint(val + k0 + pos, pa) * (double)ldx<HOT>(x, xh, ld_hint(col + k0 + pos, pa), px);
     }
     int s0 = __shfl_up_sync(0xffffffffu, e_[0], 1);
     const int last0 = __shfl_sync(0xffffffffu, e_[0], 31);
@@ -1354,7 +1354,7 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
             r = tile_ptr[n_tiles];
             if ((int64_t)rp[r] < e) {
                 const int64_t end = rp[r + 1];
-                for (int64_t k = e + lane; k < end; k += 32) s += (double)val[k] * (double)ld_x(xp<HOT>(x, xh, col[k]), px);
+                for (int64_t k = e + lane; k < end; k += 32) s += (double)val[k] * (double)ldx<HOT>(x, xh, col[k], px);
             } else {
                 r = -1;
             }
@@ -1389,7 +1389,7 @@ k_csr5(const IT *__restrict__ rp, const int *__restrict__ col, const V *__restri
     const int y_off = (int)((d >> 16) & 0x1FFu);
     double p[SIGMA];
 #pragma unroll
-    for (int s = 0; s < SIGMA; ++s) p[s] = (double)v[s] * (double)ld_x(xp<HOT>(x, xh, c[s]), px);
+    for (int s = 0; s < SIGMA; ++s) p[s] = (double)v[s] * (double)ldx<HOT>(x, xh, c[s], px);
     __syncwarp();
 
     auto emit = [&](int idx, double sum) {
