@@ -58,9 +58,36 @@ __global__ void k_hp(const int *__restrict__ col, const double *__restrict__ val
 }
 }  // namespace
 
+// hot == 3: mode 2 + an L2 access-policy window (persisting) over xhot, with `persist`
+// bytes of L2 set aside for persisting lines
+extern "C" long long hp_persist_max() {
+    int v = 0;
+    cudaDeviceGetAttribute(&v, cudaDevAttrMaxPersistingL2CacheSize, 0);
+    return v;
+}
+extern "C" int hp_set_persist(size_t bytes) {
+    return (int)cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, bytes);
+}
 extern "C" int hp_run(int hot, const int *col, const double *val, int64_t nnz, const double *x, const double *xhot, int K,
                       int blocks, int threads, double *out, void *stream) {
     cudaStream_t s = (cudaStream_t)stream;
+    if (hot == 3) {
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(blocks);
+        cfg.blockDim = dim3(threads);
+        cfg.stream = s;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeAccessPolicyWindow;
+        at[0].val.accessPolicyWindow.base_ptr = (void *)xhot;
+        at[0].val.accessPolicyWindow.num_bytes = (size_t)K * 8;
+        at[0].val.accessPolicyWindow.hitRatio = 1.0f;
+        at[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        at[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        cudaLaunchKernelEx(&cfg, k_hp<2>, col, val, nnz, x, xhot, K, out);
+        return (int)cudaGetLastError();
+    }
     size_t sm = hot == 1 ? (size_t)K * 8 : 0;
     if (hot == 1) {
         cudaFuncSetAttribute(k_hp<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);

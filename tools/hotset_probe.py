@@ -21,6 +21,7 @@ def main():
     subprocess.check_call(["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-Xcompiler", "-fPIC",
                            "-shared", os.path.join(HERE, "hotset_probe.cu"), "-o", so])
     L = ctypes.CDLL(so)
+    L.hp_set_persist.argtypes = [ctypes.c_size_t]
     L.hp_run.argtypes = [ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p,
                          ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p]
     rp, col, val = gpu.rmat(scale, seed=0x5EED0003)
@@ -56,6 +57,14 @@ def main():
         xhot = x[hot].contiguous()
         res[f"glob{K}_592x256"] = t(lambda: L.hp_run(2, enc.data_ptr(), val.data_ptr(), col.numel(), x.data_ptr(),
                                                        xhot.data_ptr(), K, 592, 256, out.data_ptr(), s.cuda_stream))
+        L.hp_persist_max.restype = ctypes.c_longlong
+        pmax = int(L.hp_persist_max())
+        res["persisting_l2_max"] = pmax
+        for frac in (0.5, 1.0):
+            L.hp_set_persist(ctypes.c_size_t(int(pmax * frac)))
+            res[f"persist{K}_{frac}"] = t(lambda: L.hp_run(3, enc.data_ptr(), val.data_ptr(), col.numel(), x.data_ptr(),
+                                                             xhot.data_ptr(), K, 592, 256, out.data_ptr(), s.cuda_stream))
+        L.hp_set_persist(ctypes.c_size_t(0))
         for blocks, threads in ((148, 1024),):
             if K * 8 * (blocks // 148) > 140 * 1024 or K > 32768:
                 continue
