@@ -47,7 +47,6 @@ constexpr int kSub = 8192;                      // diagonal items per sub-span
 constexpr int kChunk = 512;                     // nonzero positions per warp chunk (16 per lane)
 constexpr int kBmWords = (kSub + kChunk) / 32;  // row-start bitmap words per warp (+ alignment slack)
 constexpr int kSharedHist = 1024;               // row-length histogram bins kept in shared memory
-constexpr int kRowUnroll = 4;                   // row windows (32 rows) in flight per warp
 constexpr int kRowW = 4;                        // diagonal weight of a row start (a row costs ~4 nonzeros)
 
 enum : unsigned { BAD_ROWPTR_ENDS = 1, BAD_ROWPTR_ORDER = 2, BAD_COL_RANGE = 4, BAD_COL_ORDER = 8 };
@@ -229,6 +228,28 @@ k_features(const IT *__restrict__ rp, const int *__restrict__ col, int64_t n, in
     // its row-start bit is set here, so its block count is this warp's
     bool pending_rs = i0 > 0 && k0 < k1 && (int64_t)__ldg(rp + i0 - 1) == (int64_t)k0;
 
+    // row_ptr window of R1 (rows wrb .. wrb+127, four per lane, + row wrb+128), kept across sub-spans
+    const bool rp_vec = (reinterpret_cast<uintptr_t>(rp) & 15) == 0;
+    auto load_win = [&](int64_t rb, IT (&a)[4], IT &a4) {
+        const int64_t q = rb + 4 * lane;
+        if (rp_vec && q + 3 <= n) {
+            if constexpr (sizeof(IT) == 4) {
+                const int4 t = __ldg(reinterpret_cast<const int4 *>(rp + q));
+                a[0] = t.x; a[1] = t.y; a[2] = t.z; a[3] = t.w;
+            } else {
+                const longlong2 t0 = __ldg(reinterpret_cast<const longlong2 *>(rp + q));
+                const longlong2 t1 = __ldg(reinterpret_cast<const longlong2 *>(rp + q) + 1);
+                a[0] = t0.x; a[1] = t0.y; a[2] = t1.x; a[3] = t1.y;
+            }
+        } else {
+#pragma unroll
+            for (int u = 0; u < 4; ++u) a[u] = __ldg(rp + (q + u < n ? q + u : n));
+        }
+        a4 = __ldg(rp + (rb + 128 < n ? rb + 128 : n));
+    };
+    IT wa[4] = {0, 0, 0, 0}, wa4 = 0;
+    int64_t wrb = 0;
+    bool have_win = false;
     int64_t r = i0, dcur = d0;
     P kcur = k0;
     while (true) {
@@ -245,74 +266,136 @@ k_features(const IT *__restrict__ rp, const int *__restrict__ col, int64_t n, in
         // ---- R1: rows r with g(r+1) = row_ptr[r] + kRowW*(r+1) <= dsub (every row < i1 when
         //      last), taken strictly in order: lengths (sums, min/max, empty, HYB overflow,
         //      histogram), row_ptr validity, and row-start bits of their start positions.
-        //      Relative form: (row_ptr[r] - base) + kRowW*(r - r_start) <= lim.
+        //      Relative form: row_ptr[r] - base <= lim - kRowW*(r - r_start).
+        //      Windows of 128 rows from wrb = r & ~3, four consecutive rows per lane (one
+        //      16-byte load): the next window is loaded while this one is processed, and the
+        //      window a stop leaves open carries over to the next sub-span (shuffles).
         const int64_t r_start = r;
         const int64_t lim64 = dsub - kRowW * (r_start + 1) - (int64_t)base;
         const int lim = last ? INT_MAX : (int)(lim64 < INT_MIN ? INT_MIN : (lim64 > INT_MAX ? INT_MAX : lim64));
         const int64_t jmax64 = i1 - r_start;
         const int jmax = (int)(jmax64 < INT_MAX - 1024 ? jmax64 : INT_MAX - 1024);
-        while (r < i1) {
-            IT a[kRowUnroll + 1];
-#pragma unroll
-            for (int u = 0; u < kRowUnroll; ++u) {
-                const int64_t rr = r + u * 32 + lane;
-                a[u] = __ldg(rp + (rr < n ? rr : n));
+        if (r < i1) {
+            if (!have_win) {
+                wrb = r & ~(int64_t)3;
+                load_win(wrb, wa, wa4);
+                have_win = true;
             }
-            a[kRowUnroll] = __ldg(rp + (r + 32 * kRowUnroll < n ? r + 32 * kRowUnroll : n));
-            const int j0 = (int)(r - r_start);
-            int taken = 0;
-            bool stop = false;
+            while (true) {
+                IT na[4], na4;
+                load_win(wrb + 128, na, na4);
+                const int off = (int)(r - wrb);
+                const int jb = (int)(wrb - r_start) + 4 * lane;
+                P av[4], bv[4];
 #pragma unroll
-            for (int u = 0; u < kRowUnroll; ++u) {
-                const int j = j0 + u * 32 + lane;
-                const P arel = (P)(a[u] - base);
-                const bool want = j < jmax && (last || arel + (P)(kRowW * j) <= (P)lim);
-                const unsigned wm = __ballot_sync(0xffffffffu, want);
-                const int plen = stop ? 0 : (wm == 0xffffffffu ? 32 : __ffs(~wm) - 1);
-                const bool inr = lane < plen;
-                const P nx = __shfl_down_sync(0xffffffffu, a[u], 1);
-                const P nw = u + 1 < kRowUnroll ? __shfl_sync(0xffffffffu, a[u + 1 < kRowUnroll ? u + 1 : u], 0)
-                                                : a[kRowUnroll];       // first row of the next window
-                const P bb = lane == 31 ? nw : nx;
-                P len = bb - a[u];
-                if (inr) {
-                    if (arel >= (P)kc_rel && arel < (P)kCap) atomicOr(&bm[(int)arel >> 5], 1u << ((int)arel & 31));
-                    if (len < 0 || a[u] < 0 || bb > nnzP) { bad |= BAD_ROWPTR_ORDER; len = 0; }
-                    const unsigned ul = (unsigned)len;
-                    len2 += (unsigned long long)ul * ul;
-                    len_mn = min(len_mn, ul);
-                    len_mx = max(len_mx, ul);
-                    n_empty += len == 0;
-                    over += (unsigned)(len > khP ? len - khP : (P)0);
+                for (int u = 0; u < 4; ++u) av[u] = (P)wa[u];
+                const P nx = __shfl_down_sync(0xffffffffu, av[0], 1);
+                bv[0] = av[1]; bv[1] = av[2]; bv[2] = av[3];
+                bv[3] = lane == 31 ? (P)wa4 : nx;
+                int fb = 4;                                  // the lane's first unwanted row
+#pragma unroll
+                for (int u = 3; u >= 0; --u) {
+                    const int j = jb + u;
+                    const bool want = 4 * lane + u < off ||
+                                      (j < jmax && (last || av[u] - base <= (P)(lim - kRowW * j)));
+                    if (!want) fb = u;
                 }
-                if (use_hist) {                                      // empty rows: n_empty (bin 0)
-                    const bool hb = inr && len > 0;
-                    const unsigned bin = hb ? (unsigned)(len < hbinP ? len : hbinP) : 0u;
-                    const unsigned hm = __ballot_sync(0xffffffffu, hb);
-                    if (hm) {
-                        const int lead = __ffs(hm) - 1;
-                        const unsigned b0 = __shfl_sync(0xffffffffu, bin, lead);
-                        if (__all_sync(0xffffffffu, !hb || bin == b0)) {  // one length bin for the window
-                            if (lane == lead) {
-                                if ((int)b0 < sh_bins) atomicAdd(&s_hist[b0], (unsigned)__popc(hm));
-                                else atomicAdd(&hist[b0], (unsigned long long)__popc(hm));
+                const unsigned fm = __ballot_sync(0xffffffffu, fb < 4);
+                const int fl0 = fm ? __ffs(fm) - 1 : 0;
+                const int fbf = __shfl_sync(0xffffffffu, fb, fl0);
+                const int cutoff = fm ? 4 * fl0 + fbf : 128;
+                unsigned cw = UINT_MAX, cm = 0;              // row-start bits of the lane's rows
+                int hcnt = 0;
+                unsigned hbin0 = 0, binv[4];
+                bool huni = true;
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const int idx = 4 * lane + u;
+                    binv[u] = UINT_MAX;
+                    if (idx >= off && idx < cutoff) {
+                        const P arel = av[u] - base;
+                        if (arel >= (P)kc_rel && arel < (P)kCap) {
+                            const unsigned wd = (unsigned)arel >> 5, bit = 1u << ((unsigned)arel & 31);
+                            if (wd != cw) {
+                                if (cm) atomicOr(&bm[cw], cm);
+                                cw = wd;
+                                cm = 0;
                             }
-                        } else if (hb) {
-                            if ((int)bin < sh_bins) atomicAdd(&s_hist[bin], 1u);
-                            else atomicAdd(&hist[bin], 1ull);
+                            cm |= bit;
+                        }
+                        P len = bv[u] - av[u];
+                        if (len < 0 || av[u] < 0 || bv[u] > nnzP) { bad |= BAD_ROWPTR_ORDER; len = 0; }
+                        const unsigned ul = (unsigned)len;
+                        len2 += (unsigned long long)ul * ul;
+                        len_mn = min(len_mn, ul);
+                        len_mx = max(len_mx, ul);
+                        n_empty += len == 0;
+                        over += (unsigned)(len > khP ? len - khP : (P)0);
+                        if (use_hist && len > 0) {                // empty rows: n_empty (bin 0)
+                            const unsigned bin = (unsigned)(len < hbinP ? len : hbinP);
+                            binv[u] = bin;
+                            if (hcnt == 0) hbin0 = bin;
+                            else huni = huni && bin == hbin0;
+                            ++hcnt;
                         }
                     }
                 }
-                taken += plen;
-                if (plen < 32) stop = true;
+                if (cm) atomicOr(&bm[cw], cm);
+                if (use_hist) {
+                    const unsigned hm = __ballot_sync(0xffffffffu, hcnt > 0);
+                    if (hm) {
+                        const int lead = __ffs(hm) - 1;
+                        const unsigned b0 = __shfl_sync(0xffffffffu, hbin0, lead);
+                        if (__all_sync(0xffffffffu, hcnt == 0 || (huni && hbin0 == b0))) {  // one bin
+                            const unsigned tot = __reduce_add_sync(0xffffffffu, (unsigned)hcnt);
+                            if (lane == lead) {
+                                if ((int)b0 < sh_bins) atomicAdd(&s_hist[b0], tot);
+                                else atomicAdd(&hist[b0], (unsigned long long)tot);
+                            }
+                        } else {
+#pragma unroll
+                            for (int u = 0; u < 4; ++u) {
+                                if (binv[u] == UINT_MAX) continue;
+                                if ((int)binv[u] < sh_bins) atomicAdd(&s_hist[binv[u]], 1u);
+                                else atomicAdd(&hist[binv[u]], 1ull);
+                            }
+                        }
+                    }
+                }
+                r = wrb + cutoff;
+                if (cutoff < 128) {
+                    // carry: the window from r & ~3 = rows of this window and the next
+                    const int sh = cutoff >> 2;
+                    const int src = (lane + sh) & 31;
+                    const bool hi = lane + sh >= 32;
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        const IT x0 = __shfl_sync(0xffffffffu, wa[u], src);
+                        const IT x1 = __shfl_sync(0xffffffffu, na[u], src);
+                        wa[u] = hi ? x1 : x0;
+                    }
+                    wa4 = __shfl_sync(0xffffffffu, na[0], sh);
+                    wrb += 4 * sh;
+                    break;
+                }
+                wrb += 128;
+#pragma unroll
+                for (int u = 0; u < 4; ++u) wa[u] = na[u];
+                wa4 = na4;
+                if (r >= i1) break;
             }
-            r += taken;
-            if (stop) break;
         }
         const int64_t r_end = r;
         P knext = k1;
         if (!last) {
-            const int64_t rpe = (int64_t)__ldg(rp + (r_end < n ? r_end : n));
+            int64_t rpe;
+            if (have_win) {                                // window at wrb = r_end & ~3
+                const int cu = (int)(r_end - wrb);
+                const IT sel = cu == 0 ? wa[0] : cu == 1 ? wa[1] : cu == 2 ? wa[2] : wa[3];
+                rpe = (int64_t)__shfl_sync(0xffffffffu, sel, 0);
+            } else {
+                rpe = (int64_t)__ldg(rp + (r_end < n ? r_end : n));
+            }
             const int64_t kk = dsub - kRowW * r_end;
             knext = clampk(kk < rpe ? kk : rpe);
             if (knext < kcur) knext = kcur;

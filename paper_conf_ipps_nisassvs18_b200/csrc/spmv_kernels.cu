@@ -555,7 +555,11 @@ k_coo(const int *__restrict__ row, const int *__restrict__ col, const V *__restr
     const int before = k0 > 0 ? __ldg(row + k0 - 1) : -1;                  // row before the tile
     const int64_t nr = k0 + cnt < nnz ? (int64_t)__ldg(row + k0 + cnt) : n_rows;   // next tile's first row
     const int last_lane = (cnt - 1) >> 3;
-    const int rl = __shfl_sync(0xffffffffu, r[(cnt - 1) & 7], last_lane);   // tile's last row
+    int rsel = r[0];             // the lane's last valid row = max (rows sorted; no local-memory index)
+#pragma unroll
+    for (int q = 1; q < 8; ++q)
+        if (q < nv) rsel = max(rsel, r[q]);
+    const int rl = __shfl_sync(0xffffffffu, rsel, last_lane);              // tile's last row
     const bool cont = before == rf;                                        // leading continuation
     const int64_t Wlo = (!ACCUM && t == 0) ? 0 : (int64_t)rf + (cont ? 1 : 0);
     const int64_t Whi = ACCUM ? (int64_t)rl + 1 : (nr == rl ? nr + 1 : nr);
