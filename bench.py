@@ -9,6 +9,7 @@ separately, not inside the step.
 
   value  = sum over formats of 2*nnz / (time of the K timed steps / K)   [GFLOP/s]
   e2e    = the same through the public API with host x in / host y out every step
+           (spmv_run_host_multi: x and y_in cross PCIe once, every format's y comes back)
 
 Workload (``--config``): BASELINE configs[1] (lap4096: 5-point Laplacian, 4096^2 grid,
 fp64) by default at every N.  At N = 1 the line also carries configs[2] (R-MAT 24,
@@ -635,7 +636,28 @@ def run_single(args):
 
     # ---- end to end through the C ABI with pinned host buffers
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and not (args.e2e_per_call or args.e2e_serial):
+        # the label-collection call: x and y_in cross PCIe once per step for all formats,
+        # each format's result comes back (spmv_run_host_multi)
+        xnp = x.cpu().pin_memory().numpy()
+        yin = y0.cpu().pin_memory().numpy()
+        outs = [y0.cpu().pin_memory().numpy() for _ in fmts]
+        hl = [handles[f] for f in fmts]
+        e2e_steps = max(3, min(args.steps, args.e2e_steps))
+        sp.run_host_multi(hl, 1.0, xnp, 1.0, yin, outs)          # first call allocates the io buffers
+        sp.run_host_multi(hl, 1.0, xnp, 1.0, yin, outs)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(e2e_steps):
+            sp.run_host_multi(hl, 1.0, xnp, 1.0, yin, outs)
+        dt = time.perf_counter() - t0
+        V = 8 if dtype == torch.float64 else 4
+        e2e = {"value": 2.0 * dA.nnz * len(fmts) / (dt / e2e_steps) / 1e9, "unit": "GFLOP/s",
+               "h2d_bytes_per_step": (dA.n_cols + dA.n_rows) * V,
+               "d2h_bytes_per_step": len(fmts) * dA.n_rows * V, "steps": e2e_steps,
+               "api": "spmv_run_host_multi (pinned host x and y_in -> device once, every format run from a "
+                      "device copy of y_in, each result -> host while the next format runs, sync)"}
+    elif not args.no_e2e:
         xnp = x.cpu().pin_memory().numpy()
         ynps = {f: y0.cpu().pin_memory().numpy() for f in fmts}
         e2e_steps = max(3, min(args.steps, args.e2e_steps))
@@ -941,7 +963,9 @@ def main():
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo: functional check of N ranks on fewer GPUs (not a performance number)")
     ap.add_argument("--e2e-steps", type=int, default=10)
-    ap.add_argument("--e2e-serial", action="store_true", help="e2e: run the formats' host calls in turn")
+    ap.add_argument("--e2e-serial", action="store_true", help="e2e: per-format spmv_run_host calls in turn")
+    ap.add_argument("--e2e-per-call", action="store_true",
+                    help="e2e: per-format spmv_run_host calls (x/y copied per format), one host thread each")
     ap.add_argument("--feat-reps", type=int, default=20, help="warm spmv_features calls timed")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0)

@@ -190,6 +190,21 @@ spmv_status spmv_run(spmv_handle *h, const void *alpha, const void *x,
 spmv_status spmv_run_host(spmv_handle *h, const void *alpha, const void *x_host,
                           const void *beta, void *y_host, void *stream);
 
+/* Label-collection variant of spmv_run_host (every format of a
+ * matrix is timed on the same x, §IV-B): hs[0..k) are k >= 1 distinct handles of ONE
+ * matrix (same ctx, dtype, n_rows and n_cols; any formats).  x_host (n_cols) and
+ * y_in_host (n_rows; not read when beta == 0) are copied host->device ONCE; then for
+ * each i, y_i = alpha*A_i*x + beta*y_in is computed from a device copy of y_in and
+ * copied back into y_out_host[i] (n_rows values), the copy of result i overlapping run
+ * i+1 (a second, library-created stream).  Host buffers: pinned or pageable, owned by
+ * the caller, not retained.  Device buffers: x and y_in owned by hs[0], each result by
+ * its handle (allocated on first use, freed by spmv_destroy).  Synchronizes before
+ * returning; the handles must not be running elsewhere.  SPMV_ERR_INVALID_ARG for
+ * k < 1, NULL pointers, a repeated handle or handles of different shapes. */
+spmv_status spmv_run_host_multi(spmv_handle *const *hs, int k, const void *alpha, const void *x_host,
+                                const void *beta, const void *y_in_host, void *const *y_out_host,
+                                void *stream);
+
 /* Number of kernel launches one spmv_run issues for this handle (host output). */
 spmv_status spmv_run_launches(const spmv_handle *h, int *launches);
 

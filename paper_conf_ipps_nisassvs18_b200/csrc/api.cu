@@ -256,6 +256,66 @@ spmv_status spmv_run_host(spmv_handle *h, const void *alpha, const void *x_host,
     return SPMV_OK;
 }
 
+spmv_status spmv_run_host_multi(spmv_handle *const *hs, int k, const void *alpha, const void *x_host,
+                                const void *beta, const void *y_in_host, void *const *y_out_host, void *stream) {
+    if (!hs || k < 1 || !alpha || !beta || !y_out_host) { set_error("NULL handles/alpha/beta/y_out or k < 1"); return SPMV_ERR_INVALID_ARG; }
+    spmv_handle *H = hs[0];
+    if (!H) { set_error("NULL handle"); return SPMV_ERR_INVALID_ARG; }
+    for (int i = 0; i < k; ++i) {
+        const spmv_handle *h = hs[i];
+        if (!h || h->ctx != H->ctx || h->dtype != H->dtype || h->n_rows != H->n_rows || h->n_cols != H->n_cols) {
+            set_error("spmv_run_host_multi: handle " + std::to_string(i) + " is not of the first handle's ctx/dtype/shape");
+            return SPMV_ERR_INVALID_ARG;
+        }
+        for (int j = 0; j < i; ++j)
+            if (hs[j] == h) { set_error("spmv_run_host_multi: a handle appears twice"); return SPMV_ERR_INVALID_ARG; }
+        if (H->n_rows && !y_out_host[i]) { set_error("spmv_run_host_multi: NULL y_out"); return SPMV_ERR_INVALID_ARG; }
+    }
+    const size_t V = H->dtype == SPMV_F64 ? 8 : 4;
+    const double b = H->dtype == SPMV_F64 ? *(const double *)beta : *(const float *)beta;
+    if (H->n_rows && b != 0.0 && !y_in_host) { set_error("spmv_run_host_multi: NULL y_in with beta != 0"); return SPMV_ERR_INVALID_ARG; }
+    cudaStream_t s = as_stream(stream);
+    SPMV_ON_DEVICE(H->ctx->device);
+    const size_t bx = (size_t)H->n_cols * V, by = (size_t)H->n_rows * V;
+    if (!H->io_x.p && bx) { SPMV_TRY(dev_alloc(H->ctx, bx, s, &H->io_x.p)); H->io_x.bytes = bx; }
+    if (!H->io_yin.p && by && b != 0.0) { SPMV_TRY(dev_alloc(H->ctx, by, s, &H->io_yin.p)); H->io_yin.bytes = by; }
+    for (int i = 0; i < k; ++i)
+        if (!hs[i]->io_y.p && by) { SPMV_TRY(dev_alloc(H->ctx, by, s, &hs[i]->io_y.p)); hs[i]->io_y.bytes = by; }
+    // x and y_in cross PCIe once; each run starts from a device copy of y_in; run i's result
+    // goes back on a second stream while run i+1 computes
+    if (bx) SPMV_CUDA_TRY(cudaMemcpyAsync(H->io_x.p, x_host, bx, cudaMemcpyHostToDevice, s));
+    if (by && b != 0.0) SPMV_CUDA_TRY(cudaMemcpyAsync(H->io_yin.p, y_in_host, by, cudaMemcpyHostToDevice, s));
+    cudaStream_t c = nullptr;
+    SPMV_CUDA_TRY(cudaStreamCreateWithFlags(&c, cudaStreamNonBlocking));
+    std::vector<cudaEvent_t> ev((size_t)k, nullptr);
+    spmv_status st = SPMV_OK;
+    for (int i = 0; i < k && st == SPMV_OK; ++i) {
+        spmv_handle *h = hs[i];
+        if (by && b != 0.0 && cudaMemcpyAsync(h->io_y.p, H->io_yin.p, by, cudaMemcpyDeviceToDevice, s) != cudaSuccess) {
+            set_error(std::string("spmv_run_host_multi: y_in copy: ") + cudaGetErrorString(cudaGetLastError()));
+            st = SPMV_ERR_CUDA;
+            break;
+        }
+        st = spmv_run(h, alpha, H->io_x.p, beta, h->io_y.p, stream);
+        if (st != SPMV_OK || !by) continue;
+        if (cudaEventCreateWithFlags(&ev[i], cudaEventDisableTiming) != cudaSuccess || cudaEventRecord(ev[i], s) != cudaSuccess ||
+            cudaStreamWaitEvent(c, ev[i], 0) != cudaSuccess ||
+            cudaMemcpyAsync(y_out_host[i], h->io_y.p, by, cudaMemcpyDeviceToHost, c) != cudaSuccess) {
+            set_error(std::string("spmv_run_host_multi: y copy-back: ") + cudaGetErrorString(cudaGetLastError()));
+            st = SPMV_ERR_CUDA;
+        }
+    }
+    const cudaError_t e1 = cudaStreamSynchronize(c), e2 = cudaStreamSynchronize(s);
+    for (cudaEvent_t e : ev)
+        if (e) cudaEventDestroy(e);
+    cudaStreamDestroy(c);
+    if (st == SPMV_OK && (e1 != cudaSuccess || e2 != cudaSuccess)) {
+        set_error(std::string("spmv_run_host_multi: ") + cudaGetErrorString(e1 != cudaSuccess ? e1 : e2));
+        st = SPMV_ERR_CUDA;
+    }
+    return st;
+}
+
 spmv_status spmv_run_launches(const spmv_handle *h, int *launches) {
     if (!h || !launches) return SPMV_ERR_INVALID_ARG;
     *launches = run_launch_count(h, false);
@@ -357,6 +417,7 @@ spmv_status spmv_destroy(spmv_handle *h, void *stream) {
     dev_free(h->ctx, h->sched.p, h->sched.bytes, s);
     dev_free(h->ctx, h->xhot.p, h->xhot.bytes, s);
     dev_free(h->ctx, h->io_y.p, h->io_y.bytes, s);
+    dev_free(h->ctx, h->io_yin.p, h->io_yin.bytes, s);
     delete h;
     return SPMV_OK;
 }

@@ -88,6 +88,7 @@ struct spmv_handle {
     int64_t n_carry = 0;
     // spmv_run_host staging
     spmv::DevArray io_x, io_y;
+    spmv::DevArray io_yin;                   // spmv_run_host_multi: the device copy of y_in (first handle)
     // CSR-vector dynamic batch scheduler: one u64 counter, zeroed before every run
     spmv::DevArray sched;
     // hot columns (A30): the x entries stored as -2 - slot are read from xhot[slot], packed

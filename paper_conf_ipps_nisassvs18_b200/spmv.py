@@ -120,6 +120,7 @@ def lib():
                                        C.POINTER(_P)]),
             "spmv_run": (C.c_int, [_P, _P, _P, _P, _P, _P]),
             "spmv_run_host": (C.c_int, [_P, _P, _P, _P, _P, _P]),
+            "spmv_run_host_multi": (C.c_int, [C.POINTER(_P), C.c_int, _P, _P, _P, _P, C.POINTER(_P), _P]),
             "spmv_run_launches": (C.c_int, [_P, C.POINTER(C.c_int)]),
             "spmv_info": (C.c_int, [_P, C.POINTER(spmv_handle_info)]),
             "spmv_export": (C.c_int, [_P, C.c_int, _P, C.c_size_t, C.POINTER(C.c_size_t), _P]),
@@ -290,6 +291,22 @@ def spmv_convert(A: CSR, fmt, stream=None, **opts) -> "Handle":
 
 
 convert = spmv_convert
+
+
+def run_host_multi(handles, alpha, x: np.ndarray, beta, y_in: Optional[np.ndarray], y_outs, stream=None):
+    """spmv_run_host_multi: k handles of one matrix on the same host x / y_in (copied to the
+    device once), result i copied back into y_outs[i] (host arrays of n_rows)."""
+    hs = list(handles)
+    if not hs or len(y_outs) != len(hs):
+        raise ValueError("one output array per handle")
+    h0 = hs[0]
+    a, b = h0._scalar(alpha), h0._scalar(beta)
+    arr = (_P * len(hs))(*[h.ptr for h in hs])
+    outs = (_P * len(hs))(*[(y.ctypes.data if y.size else None) for y in y_outs])
+    yin = y_in.ctypes.data if (y_in is not None and y_in.size) else None
+    _check(lib().spmv_run_host_multi(arr, len(hs), C.byref(a), x.ctypes.data if x.size else None, C.byref(b),
+                                     yin, outs, _stream_ptr(stream)))
+    return y_outs
 
 
 def spmv_partition(A: CSR, nparts: int, stream=None) -> np.ndarray:

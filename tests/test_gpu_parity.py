@@ -373,6 +373,58 @@ def test_run_host_end_to_end(sp, fmt):
     assert oracle.check_tolerance(out, ref, bound, 1e-12)[0]
 
 
+@pytest.mark.parametrize("beta", [0.5, 0.0], ids=["beta", "beta0"])
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32], ids=["f64", "f32"])
+@pytest.mark.parametrize("name", ["rmat12", "lap37", "sparse_rows", "nnz0_rows5"])
+def test_run_host_multi(sp, name, dtype, beta):
+    """spmv_run_host_multi (x and y_in cross PCIe once for all formats): every result
+    is bit-identical to the handle's own spmv_run on device buffers and within the bound
+    of the oracle; y_in is left untouched (and not read when beta == 0)."""
+    kind = "f64" if dtype == torch.float64 else "f32"
+    A = case(name, kind)
+    dA = to_dev(sp, A, dtype)
+    hs, fmts = [], []
+    for f in sp.PAPER_FORMATS:
+        try:
+            hs.append(sp.convert(dA, f))
+            fmts.append(f)
+        except sp.SpmvError as e:
+            assert e.status == 3
+    npd = np.float64 if dtype == torch.float64 else np.float32
+    x = matgen.vector(A.n_cols, 6, 1).astype(npd)
+    y0 = matgen.vector(A.n_rows, 6, 2).astype(npd)
+    y_in = None if beta == 0.0 else y0.copy()
+    outs = [np.full(A.n_rows, np.nan, npd) for _ in hs]
+    sp.run_host_multi(hs, 1.5, x, beta, y_in, outs)
+    if y_in is not None:
+        assert np.array_equal(y_in, y0)
+    ref, bound = oracle.spmv_csr(A, x.astype(np.float64), 1.5, beta, y0.astype(np.float64), with_bound=True)
+    tol = 1e-12 if dtype == torch.float64 else 1e-5
+    xd = torch.from_numpy(x).cuda()
+    for f, h, out in zip(fmts, hs, outs):
+        yd = torch.from_numpy(y0).cuda() if beta != 0.0 else torch.full((A.n_rows,), float("nan"), dtype=dtype, device="cuda")
+        h.run(1.5, xd, beta, yd)
+        torch.cuda.synchronize()
+        assert np.array_equal(yd.cpu().numpy(), out), f
+        assert oracle.check_tolerance(out.astype(np.float64), ref, bound, tol)[0], f
+
+
+def test_run_host_multi_errors(sp):
+    A, B = case("rmat12", "f64"), case("lap37", "f64")
+    hA = sp.convert(to_dev(sp, A, torch.float64), "csr")
+    hB = sp.convert(to_dev(sp, B, torch.float64), "csr")
+    x = matgen.vector(A.n_cols, 1, 1)
+    y = matgen.vector(A.n_rows, 1, 2)
+    out = [np.zeros(A.n_rows), np.zeros(A.n_rows)]
+    for hs in ([hA, hB], [hA, hA]):
+        with pytest.raises(sp.SpmvError) as e:
+            sp.run_host_multi(hs, 1.0, x, 1.0, y, out)
+        assert e.value.status == 1
+    with pytest.raises(sp.SpmvError) as e:                 # beta != 0 needs y_in
+        sp.run_host_multi([hA], 1.0, x, 1.0, None, out[:1])
+    assert e.value.status == 1
+
+
 @pytest.mark.parametrize("dtype", [torch.float64, torch.float32], ids=["f64", "f32"])
 @pytest.mark.parametrize("fmt", ("csr", "merge", "csr5", "coo", "hyb", "ell"))
 def test_long_sequential_stress(sp, fmt, dtype):
