@@ -81,7 +81,12 @@ __global__ void k_scale(V *y, int64_t n, double beta) {
 // even when rows are as short as the 5-point stencil's.  Rows longer than W finish
 // with the whole warp on one row at a time (8 loads per lane in flight, accumulators
 // folded every kFold steps, A13) -- the paper's warp-per-row kernel for long rows.
-template <int W> struct VecCfg { static constexpr int U = W <= 8 ? 32 / (32 / W) : (W == 16 ? 4 : 2); };
+// fp64 at W = 16: 16 rows per group (a 32-row batch, one claim of the dynamic scheduler at
+// a time) -- R-MAT 24 CSR 1.81 -> 1.60 ms (U = 4: 1.81, 8: 1.72); fp32 keeps U = 4 (U = 8 /
+// 16: 1.62 / 1.76 against 1.60 ms)
+template <int W, typename V = double> struct VecCfg {
+    static constexpr int U = W <= 8 ? 32 / (32 / W) : (W == 16 ? (sizeof(V) == 8 ? 16 : 4) : 2);
+};
 
 template <typename V, typename IT, int W, bool B0, int MB, bool CHUNKED, bool DYN = false, bool HOT = false>
 __global__ void __launch_bounds__(kT, MB)
@@ -89,7 +94,7 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
              const V *__restrict__ x, const V *__restrict__ xh, V *__restrict__ y, int64_t n, double alpha, double beta, int64_t long_len,
              unsigned long long *__restrict__ sched = nullptr) {
     constexpr int G = 32 / W;
-    constexpr int U = (VecCfg<W>::U * G > 32) ? 32 / G : VecCfg<W>::U;
+    constexpr int U = (VecCfg<W, V>::U * G > 32) ? 32 / G : VecCfg<W, V>::U;
     constexpr int R = G * U;                      // rows per warp iteration (<= 32)
     const int lane = threadIdx.x & 31;
     const int sub = lane & (W - 1);
@@ -100,9 +105,10 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
     // DYN: warps take groups of kDynGroup batches from a global counter (zeroed before
     // the launch), the next group requested one group ahead -- balances skewed rows (a
     // static grid stride left R-MAT warps idle behind the slowest batch sequences)
-    // (batches per group: fp64 2, fp32 4 -- R-MAT 24 fp64 group 4 1.82 ms, 2 1.79, 8 1.84;
-    // fp32 group 4 1.60, 2 1.70; R-MAT 22 fp64 0.50 / 0.47 / 0.56)
-    constexpr int kDynGroup = sizeof(V) == 8 ? 2 : 4;
+    // (batches per group: fp64 1 of 32 rows, fp32 4 of 8 rows -- R-MAT 24 fp64 with 8-row
+    // batches: group 4 1.82 ms, 2 1.79, 8 1.84, with 32-row batches: group 2 1.67, 1 1.60;
+    // fp32 group 4 1.60, 2 1.70)
+    constexpr int kDynGroup = sizeof(V) == 8 ? 1 : 4;
     unsigned long long ng = 0;
     int j = 0;
     int64_t base = gwarp * R;
