@@ -102,185 +102,257 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
     const int64_t gwarp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const uint64_t pa = policy_evict_first(), px = policy_evict_last();
-    // DYN: warps take groups of kDynGroup batches from a global counter (zeroed before
-    // the launch), the next group requested one group ahead -- balances skewed rows (a
-    // static grid stride left R-MAT warps idle behind the slowest batch sequences)
-    // (batches per group: fp64 1 of 32 rows, fp32 4 of 8 rows -- R-MAT 24 fp64 with 8-row
-    // batches: group 4 1.82 ms, 2 1.79, 8 1.84, with 32-row batches: group 2 1.67, 1 1.60;
-    // fp32 group 4 1.60, 2 1.70)
-    constexpr int kDynGroup = sizeof(V) == 8 ? 1 : 4;
-    unsigned long long ng = 0;
-    int j = 0;
-    int64_t base = gwarp * R;
-    if constexpr (DYN) {
-        unsigned long long g0 = 0;
+    // one batch of R rows: group g's U rows have nonzeros [a[u], b[u]); lane i < R holds
+    // row i's range [my_a, my_e) (slot_ok: a live row) for the long-row walk; the writer
+    // lane (sub < U) of each row writes y[my_row] (row_ok)
+    auto batch = [&](const IT (&a)[U], const IT (&b)[U], const IT ra0, const IT rhi, const bool contiguous,
+                     const bool slot_ok, const int64_t my_row, const bool row_ok) {
+            // the y value this lane will write (writer lane sub == u of group g)
+            const double yv = (!B0 && sub < U && row_ok) ? (double)y[my_row] : 0.0;
+            // first W elements of every row, all loads issued together
+            int c0[U];
+            V v0[U];
+    #pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int64_t k = (int64_t)a[u] + sub;
+                c0[u] = k < b[u] ? ld_hint(col + k, pa) : -1;
+                v0[u] = k < b[u] ? ld_hint(val + k, pa) : (V)0;
+            }
+            double s[U];
+    #pragma unroll
+            for (int u = 0; u < U; ++u) s[u] = c0[u] != -1 ? (double)v0[u] * (double)ldx<HOT>(x, xh, c0[u], px) : 0.0;
+            // the group's U results: lane sub == u of group g writes row u*G + g
+            double mine = 0.0;
+            {
+                // lane bits >= U do not index rows: plain butterflies over them; then a
+                // transpose reduction over the low bits -- at offset o a lane keeps the half
+                // of its partial sums selected by (sub & o) and adds the other half received
+                // from lane sub ^ o, so lane sub ends with row (sub mod U)'s sum (U - 1
+                // shuffles instead of a butterfly per row, U * log2(U))
+    #pragma unroll
+                for (int o = W / 2; o >= U; o >>= 1) {
+    #pragma unroll
+                    for (int u = 0; u < U; ++u) s[u] += __shfl_xor_sync(0xffffffffu, s[u], o);
+                }
+    #pragma unroll
+                for (int o = U / 2; o > 0; o >>= 1) {
+                    const bool hi = (sub & o) != 0;
+    #pragma unroll
+                    for (int j = 0; j < o; ++j) {
+                        const double send = hi ? s[j] : s[j + o];
+                        const double keep = hi ? s[j + o] : s[j];
+                        s[j] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+                    }
+                }
+                mine = s[0];
+            }
+            // rows longer than W: the remainder is processed by the WHOLE warp, one row at a
+            // time (the paper's warp-per-row vector kernel), 8 loads per lane in
+            // flight, accumulators folded every kFold steps (A13); lane i holds row i's range
+            {
+                // lane i's row range, derived only here: contiguous batches hold row starts
+                // (the batch end in rhi), compacted ones hold [start, end) directly
+                const IT my_a = ra0;
+                const IT nx = __shfl_sync(0xffffffffu, ra0, (lane + 1) & 31);
+                const IT my_e = contiguous ? (lane + 1 < R ? nx : rhi) : rhi;
+                const int64_t my_len = (int64_t)my_e - (int64_t)my_a;
+                const bool is_long = slot_ok && my_len > W && (!CHUNKED || my_len <= long_len);
+                // remainders of at most kSubMax: all such rows of the batch at once, a subgroup
+                // of SW = 32 / next_pow2(count) lanes per row, 8 predicated loads per lane per
+                // step -- one gather round trip for the batch instead of one per row (R-MAT's
+                // many rows a little longer than W)
+                const unsigned few = __ballot_sync(0xffffffffu, is_long && my_len - W <= kSubMax);
+                unsigned more = __ballot_sync(0xffffffffu, is_long) & ~few;
+                if (few) {
+                    const int nl = __popc(few);
+                    const int lg = nl > 1 ? 32 - __clz(nl - 1) : 0;
+                    const int SW = 32 >> lg;
+                    const int sg = lane >> (5 - lg), sl = lane & (SW - 1);
+                    const int ri = sg < nl ? (int)__fns(few, 0, sg + 1) : 0;
+                    const int64_t ra = (int64_t)__shfl_sync(0xffffffffu, my_a, ri) + W;
+                    const int64_t re = (int64_t)__shfl_sync(0xffffffffu, my_e, ri);
+                    const int64_t rb = sg < nl ? re : ra;
+                    double acc[8];
+    #pragma unroll
+                    for (int q = 0; q < 8; ++q) acc[q] = 0.0;
+                    for (int64_t k = ra + sl; k < rb; k += 8 * SW) {
+                        int d[8];
+                        V w[8];
+    #pragma unroll
+                        for (int q = 0; q < 8; ++q) {
+                            const bool in = k + q * SW < rb;
+                            d[q] = in ? ld_hint(col + k + q * SW, pa) : -1;
+                            w[q] = in ? ld_hint(val + k + q * SW, pa) : (V)0;
+                        }
+    #pragma unroll
+                        for (int q = 0; q < 8; ++q) if (d[q] != -1) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
+                    }
+                    double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
+                    for (int o = SW >> 1; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+                    const int wi = g * U + (sub < U ? sub : 0);           // this lane's row (writer lanes)
+                    const bool wmine = sub < U && ((few >> wi) & 1u);
+                    const int src = (__popc(few & ((1u << wi) - 1u)) << (5 - lg)) & 31;
+                    const double got = __shfl_sync(0xffffffffu, part, src);
+                    if (wmine) mine += got;
+                }
+                while (more) {
+                    const int i = __ffs(more) - 1;
+                    more &= more - 1;
+                    const int64_t ra = (int64_t)__shfl_sync(0xffffffffu, my_a, i) + W;
+                    const int64_t rb = (int64_t)__shfl_sync(0xffffffffu, my_e, i);
+                    double tot = 0.0, acc[8];
+    #pragma unroll
+                    for (int q = 0; q < 8; ++q) acc[q] = 0.0;
+                    int it = 0;
+                    int64_t k = ra + lane;
+                    for (; k + 7 * 32 < rb; k += 8 * 32) {
+                        int d[8];
+                        V w[8];
+    #pragma unroll
+                        for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
+    #pragma unroll
+                        for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
+                        if (++it == kFold) {                 // blocked summation (A13)
+    #pragma unroll
+                            for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
+                            it = 0;
+                        }
+                    }
+                    for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ldx<HOT>(x, xh, ld_hint(col + k, pa), px);
+                    double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
+                    part = warp_sum(tot + part);
+                    const int writer = (i / U) * W + i % U;   // lane holding row i's group sum
+                    if (lane == writer) mine += part;
+                }
+            }
+            if (sub < U && row_ok) {
+                double o = alpha * mine;
+                if (!B0) o = fma(beta, yv, o);
+                y[my_row] = (V)o;
+            }
+    };
+    // DYN: warps take work from a global counter (zeroed before the launch), the next
+    // claim requested one claim ahead -- balances skewed rows (a static grid stride left
+    // R-MAT warps idle behind the slowest batch sequences).
+    // fp32: a claim is a window of 64 rows whose rows with work (non-empty, not chunked)
+    // are compacted into batches of R, so that a batch never spends its lanes on empty rows
+    // (R-MAT: 57% of the rows); rows without work get beta*y (nothing to write when
+    // beta == 1).  R-MAT 24 fp32 CSR 1.60 -> 1.40 ms.  fp64 keeps contiguous 32-row
+    // batches, one per claim: compacted it measured 1.90 / 2.04 / 2.12 ms at 8 / 16 / 32-row
+    // batches against 1.58.
+    if constexpr (DYN && sizeof(V) == 4) {
+        constexpr int WIN = 64;
+        __shared__ int64_t s_row_all[kT / 32][WIN];
+        __shared__ IT s_a_all[kT / 32][WIN], s_e_all[kT / 32][WIN];
+        const int wid = threadIdx.x >> 5;
+        int64_t *s_row = s_row_all[wid];
+        IT *s_a = s_a_all[wid], *s_e = s_e_all[wid];
+        unsigned long long g0 = 0, ng = 0;
         if (lane == 0) { g0 = atomicAdd(sched, 1ull); ng = atomicAdd(sched, 1ull); }
-        base = (int64_t)__shfl_sync(0xffffffffu, g0, 0) * (kDynGroup * R);
-    }
-    IT nlo = 0, nhi = 0;                          // row pointers of the next batch (prefetched)
-    if (base < n) {
-        nlo = __ldg(rp + (base + lane < n ? base + lane : n));
-        nhi = __ldg(rp + (base + R < n ? base + R : n));
-    }
-    while (base < n) {
-        const IT rp_lo = nlo, rp_hi = nhi;
-        int64_t nb = base + nwarps * R;
+        int64_t wb = (int64_t)__shfl_sync(0xffffffffu, g0, 0) * WIN;
+        IT q0 = 0, q1 = 0, q2 = 0;                    // row pointers of the next window (prefetched)
+        auto load_win = [&](int64_t w0) {
+            q0 = __ldg(rp + (w0 + lane < n ? w0 + lane : n));
+            q1 = __ldg(rp + (w0 + 32 + lane < n ? w0 + 32 + lane : n));
+            q2 = __ldg(rp + (w0 + WIN < n ? w0 + WIN : n));
+        };
+        if (wb < n) load_win(wb);
+        while (wb < n) {
+            const IT p0 = q0, p1 = q1, p2 = q2;
+            const int64_t nb = (int64_t)__shfl_sync(0xffffffffu, ng, 0) * WIN;
+            if (lane == 0) ng = atomicAdd(sched, 1ull);
+            if (nb < n) load_win(nb);
+            const IT n0 = __shfl_down_sync(0xffffffffu, p0, 1), n1 = __shfl_down_sync(0xffffffffu, p1, 1);
+            const IT f1 = __shfl_sync(0xffffffffu, p1, 0);
+            const IT e0 = lane == 31 ? f1 : n0, e1 = lane == 31 ? p2 : n1;
+            const int64_t r0 = wb + lane, r1 = wb + 32 + lane;
+            const int64_t l0 = (int64_t)e0 - (int64_t)p0, l1 = (int64_t)e1 - (int64_t)p1;
+            const bool v0 = r0 < n, v1 = r1 < n;
+            const bool w0 = v0 && l0 > 0 && (!CHUNKED || l0 <= long_len);
+            const bool w1 = v1 && l1 > 0 && (!CHUNKED || l1 <= long_len);
+            if (beta != 1.0) {                            // empty rows and chunked rows (A25)
+                if (v0 && !w0) y_beta<V, B0>(y, r0, beta);
+                if (v1 && !w1) y_beta<V, B0>(y, r1, beta);
+            }
+            const unsigned m0 = __ballot_sync(0xffffffffu, w0), m1 = __ballot_sync(0xffffffffu, w1);
+            const int c0 = __popc(m0), T = c0 + __popc(m1);
+            const unsigned lt = (1u << lane) - 1u;
+            __syncwarp();                                 // the previous window's slots are consumed
+            if (w0) { const int sl = __popc(m0 & lt); s_row[sl] = r0; s_a[sl] = p0; s_e[sl] = e0; }
+            if (w1) { const int sl = c0 + __popc(m1 & lt); s_row[sl] = r1; s_a[sl] = p1; s_e[sl] = e1; }
+            __syncwarp();
+            for (int off = 0; off < T; off += R) {
+                const bool ok = lane < R && off + lane < T;
+                const int64_t my_r = ok ? s_row[off + lane] : 0;
+                const IT my_a = ok ? s_a[off + lane] : (IT)0, my_e = ok ? s_e[off + lane] : (IT)0;
+                IT a[U], b[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    a[u] = __shfl_sync(0xffffffffu, my_a, g * U + u);
+                    b[u] = __shfl_sync(0xffffffffu, my_e, g * U + u);
+                }
+                const int ws = g * U + (sub < U ? sub : 0);
+                const int64_t my_row = __shfl_sync(0xffffffffu, my_r, ws);
+                batch(a, b, my_a, my_e, false, ok, my_row, sub < U && off + ws < T);
+            }
+            wb = nb;
+        }
+    } else {
+        // claims of kDynGroup consecutive batches (fp64: 1 batch of 32 rows; R-MAT 24 with
+        // 8-row batches: group 4 1.82 ms, 2 1.79, 8 1.84; 32-row batches: group 2 1.67, 1 1.60)
+        constexpr int kDynGroup = sizeof(V) == 8 ? 1 : 4;
+        unsigned long long ng = 0;
+        int j = 0;
+        int64_t base = gwarp * R;
         if constexpr (DYN) {
-            if (++j < kDynGroup) {
-                nb = base + R;
-            } else {
-                j = 0;
-                nb = (int64_t)__shfl_sync(0xffffffffu, ng, 0) * (kDynGroup * R);
-                if (lane == 0) ng = atomicAdd(sched, 1ull);
-            }
+            unsigned long long g0 = 0;
+            if (lane == 0) { g0 = atomicAdd(sched, 1ull); ng = atomicAdd(sched, 1ull); }
+            base = (int64_t)__shfl_sync(0xffffffffu, g0, 0) * (kDynGroup * R);
         }
-        if (nb < n) {                             // issue the next batch's row pointers now
-            nlo = __ldg(rp + (nb + lane < n ? nb + lane : n));
-            nhi = __ldg(rp + (nb + R < n ? nb + R : n));
+        IT nlo = 0, nhi = 0;                          // row pointers of the next batch (prefetched)
+        if (base < n) {
+            nlo = __ldg(rp + (base + lane < n ? base + lane : n));
+            nhi = __ldg(rp + (base + R < n ? base + R : n));
         }
-        // group g owns the U consecutive rows g*U + u of the batch, so b[u] = a[u+1]:
-        // U + 1 shuffles of the batch's row pointers (a row per group slot u*G + g took 2U)
-        auto row_of = [&](int gg, int u) -> int { return gg * U + u; };
-        IT a[U], b[U];
-        {
-            IT e[U + 1];
-#pragma unroll
-            for (int u = 0; u <= U; ++u) {
-                const int i = g * U + u;
-                const IT t = __shfl_sync(0xffffffffu, rp_lo, i & 31);
-                e[u] = i < R ? t : rp_hi;
-            }
-#pragma unroll
-            for (int u = 0; u < U; ++u) { a[u] = e[u]; b[u] = e[u + 1]; }
-        }
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-            if (base + row_of(g, u) >= n) { a[u] = 0; b[u] = 0; }
-            if (CHUNKED && (int64_t)b[u] - (int64_t)a[u] > long_len) b[u] = a[u];   // chunked long row (A25): beta*y here
-        }
-        // the y value this lane will write (writer lane sub == u of group g: row row_of(g, u))
-        const int64_t my_row = base + row_of(g, sub < U ? sub : 0);
-        const double yv = (!B0 && sub < U && my_row < n) ? (double)y[my_row] : 0.0;
-        // first W elements of every row, all loads issued together
-        int c0[U];
-        V v0[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-            const int64_t k = (int64_t)a[u] + sub;
-            c0[u] = k < b[u] ? ld_hint(col + k, pa) : -1;
-            v0[u] = k < b[u] ? ld_hint(val + k, pa) : (V)0;
-        }
-        double s[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) s[u] = c0[u] != -1 ? (double)v0[u] * (double)ldx<HOT>(x, xh, c0[u], px) : 0.0;
-        // the group's U results: lane sub == u of group g writes row u*G + g
-        double mine = 0.0;
-        {
-            // lane bits >= U do not index rows: plain butterflies over them; then a
-            // transpose reduction over the low bits -- at offset o a lane keeps the half
-            // of its partial sums selected by (sub & o) and adds the other half received
-            // from lane sub ^ o, so lane sub ends with row (sub mod U)'s sum (U - 1
-            // shuffles instead of a butterfly per row, U * log2(U))
-#pragma unroll
-            for (int o = W / 2; o >= U; o >>= 1) {
-#pragma unroll
-                for (int u = 0; u < U; ++u) s[u] += __shfl_xor_sync(0xffffffffu, s[u], o);
-            }
-#pragma unroll
-            for (int o = U / 2; o > 0; o >>= 1) {
-                const bool hi = (sub & o) != 0;
-#pragma unroll
-                for (int j = 0; j < o; ++j) {
-                    const double send = hi ? s[j] : s[j + o];
-                    const double keep = hi ? s[j + o] : s[j];
-                    s[j] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+        while (base < n) {
+            const IT rp_lo = nlo, rp_hi = nhi;
+            int64_t nb = base + nwarps * R;
+            if constexpr (DYN) {
+                if (++j < kDynGroup) {
+                    nb = base + R;
+                } else {
+                    j = 0;
+                    nb = (int64_t)__shfl_sync(0xffffffffu, ng, 0) * (kDynGroup * R);
+                    if (lane == 0) ng = atomicAdd(sched, 1ull);
                 }
             }
-            mine = s[0];
-        }
-        // rows longer than W: the remainder is processed by the WHOLE warp, one row at a
-        // time (the paper's warp-per-row vector kernel), 8 loads per lane in
-        // flight, accumulators folded every kFold steps (A13); lane i holds row i's range
-        {
-            const IT my_a = rp_lo;
-            const IT my_b = __shfl_sync(0xffffffffu, rp_lo, (lane + 1) & 31);
-            const IT my_e = lane + 1 < R ? my_b : rp_hi;
-            const int64_t my_len = (int64_t)my_e - (int64_t)my_a;
-            const bool is_long = lane < R && base + lane < n && my_len > W && (!CHUNKED || my_len <= long_len);
-            // remainders of at most kSubMax: all such rows of the batch at once, a subgroup
-            // of SW = 32 / next_pow2(count) lanes per row, 8 predicated loads per lane per
-            // step -- one gather round trip for the batch instead of one per row (R-MAT's
-            // many rows a little longer than W)
-            const unsigned few = __ballot_sync(0xffffffffu, is_long && my_len - W <= kSubMax);
-            unsigned more = __ballot_sync(0xffffffffu, is_long) & ~few;
-            if (few) {
-                const int nl = __popc(few);
-                const int lg = nl > 1 ? 32 - __clz(nl - 1) : 0;
-                const int SW = 32 >> lg;
-                const int sg = lane >> (5 - lg), sl = lane & (SW - 1);
-                const int ri = sg < nl ? (int)__fns(few, 0, sg + 1) : 0;
-                const int64_t ra = (int64_t)__shfl_sync(0xffffffffu, my_a, ri) + W;
-                const int64_t re = (int64_t)__shfl_sync(0xffffffffu, my_e, ri);
-                const int64_t rb = sg < nl ? re : ra;
-                double acc[8];
-#pragma unroll
-                for (int q = 0; q < 8; ++q) acc[q] = 0.0;
-                for (int64_t k = ra + sl; k < rb; k += 8 * SW) {
-                    int d[8];
-                    V w[8];
-#pragma unroll
-                    for (int q = 0; q < 8; ++q) {
-                        const bool in = k + q * SW < rb;
-                        d[q] = in ? ld_hint(col + k + q * SW, pa) : -1;
-                        w[q] = in ? ld_hint(val + k + q * SW, pa) : (V)0;
-                    }
-#pragma unroll
-                    for (int q = 0; q < 8; ++q) if (d[q] != -1) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
-                }
-                double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
-                for (int o = SW >> 1; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
-                const int wi = g * U + (sub < U ? sub : 0);           // this lane's row (writer lanes)
-                const bool wmine = sub < U && ((few >> wi) & 1u);
-                const int src = (__popc(few & ((1u << wi) - 1u)) << (5 - lg)) & 31;
-                const double got = __shfl_sync(0xffffffffu, part, src);
-                if (wmine) mine += got;
+            if (nb < n) {                             // issue the next batch's row pointers now
+                nlo = __ldg(rp + (nb + lane < n ? nb + lane : n));
+                nhi = __ldg(rp + (nb + R < n ? nb + R : n));
             }
-            while (more) {
-                const int i = __ffs(more) - 1;
-                more &= more - 1;
-                const int64_t ra = (int64_t)__shfl_sync(0xffffffffu, my_a, i) + W;
-                const int64_t rb = (int64_t)__shfl_sync(0xffffffffu, my_e, i);
-                double tot = 0.0, acc[8];
+            // group g owns the U consecutive rows g*U + u of the batch, so b[u] = a[u+1]:
+            // U + 1 shuffles of the batch's row pointers (a row per group slot u*G + g took 2U)
+            IT a[U], b[U];
+            {
+                IT e[U + 1];
 #pragma unroll
-                for (int q = 0; q < 8; ++q) acc[q] = 0.0;
-                int it = 0;
-                int64_t k = ra + lane;
-                for (; k + 7 * 32 < rb; k += 8 * 32) {
-                    int d[8];
-                    V w[8];
-#pragma unroll
-                    for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
-#pragma unroll
-                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
-                    if (++it == kFold) {                 // blocked summation (A13)
-#pragma unroll
-                        for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
-                        it = 0;
-                    }
+                for (int u = 0; u <= U; ++u) {
+                    const int i = g * U + u;
+                    const IT t = __shfl_sync(0xffffffffu, rp_lo, i & 31);
+                    e[u] = i < R ? t : rp_hi;
                 }
-                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ldx<HOT>(x, xh, ld_hint(col + k, pa), px);
-                double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
-                part = warp_sum(tot + part);
-                const int writer = (i / U) * W + i % U;   // lane holding row i's group sum
-                if (lane == writer) mine += part;
+#pragma unroll
+                for (int u = 0; u < U; ++u) { a[u] = e[u]; b[u] = e[u + 1]; }
             }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                if (base + g * U + u >= n) { a[u] = 0; b[u] = 0; }
+                if (CHUNKED && (int64_t)b[u] - (int64_t)a[u] > long_len) b[u] = a[u];   // chunked long row (A25): beta*y here
+            }
+            const int64_t my_row = base + g * U + (sub < U ? sub : 0);
+            batch(a, b, rp_lo, rp_hi, true, lane < R && base + lane < n, my_row, my_row < n);
+            base = nb;
         }
-        if (sub < U && my_row < n) {
-            double o = alpha * mine;
-            if (!B0) o = fma(beta, yv, o);
-            y[my_row] = (V)o;
-        }
-        base = nb;
     }
     // PDL after k_csr_chunks (chunked handles only): exit only once the chunk grid is
     // done.  Not compiled into the unchunked kernels: even with nothing to wait for it
