@@ -50,6 +50,35 @@ def test_full_size_rmat24_fp32_general(sp):
         assert ok, (fmt, nbad, ratio)
 
 
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32], ids=["f64", "f32"])
+@pytest.mark.parametrize("beta", [0.0, 1.0, -0.5], ids=["beta0", "beta1", "beta"])
+def test_dynamic_csr_rows_every_row(sp, dtype, beta):
+    """The CSR-vector kernel's dynamically scheduled paths (>= 1.82M rows: fp64 contiguous
+    32-row batches, fp32 compacted 64-row windows; long rows chunked, A25) on R-MAT 21
+    (2.1M rows, 58% empty, rows up to 10^4): every row within the bound against the oracle,
+    for beta = 0 (y write-only, NaN on entry: empty and chunked rows must become 0), 1
+    (nothing written for rows without work) and -0.5 (beta*y for them)."""
+    from matgen import gpu
+    kind = "f64" if dtype == torch.float64 else "f32"
+    rp, col, val = gpu.rmat(21, seed=21, kind=kind, dtype=dtype)
+    n = rp.numel() - 1
+    assert n >= 1_820_000 and int((rp[1:] - rp[:-1]).max()) > 1024
+    dA = sp.CSR(rp.to(torch.int32), col, val, (n, n))
+    A = matgen.HostCSR(rp.cpu().numpy(), col.cpu().numpy(), val.cpu().double().numpy(), n, n)
+    x = gpu.vector(n, 21, 1, kind, dtype)
+    y = gpu.vector(n, 21, 2, kind, dtype)
+    ref, bound = oracle.spmv_csr(A, x.cpu().double().numpy(), 1.5, beta, y.cpu().double().numpy(), with_bound=True)
+    h = sp.convert(dA, "csr")
+    assert h.info()["csr_chunks"] > 0
+    yd = torch.full_like(y, float("nan")) if beta == 0.0 else y.clone()
+    h.run(1.5, x, beta, yd)
+    torch.cuda.synchronize()
+    out = yd.cpu().double().numpy()
+    assert np.isfinite(out).all()
+    ok, ratio, nbad = oracle.check_tolerance(out, ref, bound, 1e-12 if dtype == torch.float64 else 1e-5)
+    assert ok, (nbad, ratio)
+
+
 def _sample_rows(rp_host, n, k, seed):
     """k random rows, the 64 longest rows and the last rows (empty-row stretches)."""
     rng = np.random.default_rng(seed)
