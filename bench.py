@@ -321,7 +321,7 @@ def run_reference(args):
               f"sample)")
     line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "GFLOP/s", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
-            "higher_is_better": True, "scaling": "strong" if ws > 1 else "weak", "vs_baseline": None,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": args.dtype, "data": "synthetic",
             "config": {"workload": config, "desc": CONFIGS.get(config, {}).get("desc", config)},
             "cpu_baseline": {"value": val, "unit": "GFLOP/s", "cores": len(R.blocks), "kind": "oracle",
@@ -708,7 +708,9 @@ def run_single(args):
 
     line = {
         "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": 1, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+        # the same fixed matrix at every N (N > 1 splits its rows): strong scaling
+        "scaling": "strong",
         "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
         "config": {"workload": config, "desc": CONFIGS.get(config, {}).get("desc", config),
                    "n_rows": dA.n_rows, "n_cols": dA.n_cols, "nnz": dA.nnz, "formats": fmts,
