@@ -342,6 +342,22 @@ spmv_status spmv_halo_colmap(spmv_ctx *ctx, const spmv_csr *A, const int64_t *ro
 spmv_status spmv_gather(spmv_ctx *ctx, spmv_dtype dtype, const void *src, const int32_t *idx, int64_t n,
                         void *dst, void *stream);
 
+/* dst[idx[q]] = src[q] for q < n (DEVICE arrays of `dtype`; the idx[q] distinct, else which
+ * write lands is unspecified): the inverse of spmv_gather, used to put a compressed-row
+ * block's results back into the rank's y slice (A33).  Asynchronous. */
+spmv_status spmv_scatter(spmv_ctx *ctx, spmv_dtype dtype, const void *src, const int32_t *idx, int64_t n,
+                         void *dst, void *stream);
+
+/* Compressed rows of A (A33; DESIGN.md §7 -- a rank's foreign-column block of a banded
+ * matrix holds a few thousand non-empty rows among millions): rows_out (DEVICE int32,
+ * capacity n_rows) receives the indices of A's non-empty rows in increasing order and
+ * rp_out (DEVICE, A's ptr_type, capacity n_rows + 1) their row starts followed by nnz, so
+ * that (rp_out, A.col_idx, A.val) is the CSR of those rows; *count_host = their number.
+ * Buffers owned by the caller.  Blocks on `stream` (one readback).  SPMV_ERR_INVALID_ARG
+ * for NULL outputs or more than 2^31 - 1 rows. */
+spmv_status spmv_compress_rows(spmv_ctx *ctx, const spmv_csr *A, void *stream, int32_t *rows_out,
+                               void *rp_out, int64_t *count_host);
+
 /* ---- diagnostics ----------------------------------------------------------- */
 const char *spmv_status_str(spmv_status s);
 const char *spmv_last_error(void);

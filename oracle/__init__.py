@@ -78,6 +78,7 @@ def lib():
             "ora_csr2hyb": (C.c_int, [_i64, _p, _p, _p, _i64, _i64, _p, _p, _p, _p, _p]),
             "ora_merge_ntiles": (_i64, [_i64, _i64, _i64]),
             "ora_csr_chunks": (_i64, [_i64, _p, _i64, _p, _p]),
+            "ora_compress_rows": (_i64, [_i64, _p, _p, _p]),
             "ora_merge_coords": (C.c_int, [_i64, _p, _i64, _p, _p]),
             "ora_merge_class": (C.c_int, [_i64, _p, _i64, _i64, _i64, _p]),
             "ora_csr5_sigma": (_i64, [_i64, _i64]),
@@ -245,6 +246,17 @@ def csr_chunks(A, C):
     cr, cl = _buf(max(m, 1), np.int64), _buf(max(m, 1), np.int64)
     lib().ora_csr_chunks(A.n_rows, _ptr(A.row_ptr), int(C), _ptr(cr), _ptr(cl))
     return cr[:m], cl[:m]
+
+
+def compress_rows(A):
+    """Compressed rows (A33): (rows, rp) int64 arrays -- A's non-empty rows and their row
+    starts followed by nnz."""
+    A = CSR.of(A)
+    m = int(lib().ora_compress_rows(A.n_rows, _ptr(A.row_ptr), None, None))
+    assert m >= 0
+    rows, rp = _buf(max(m, 1), np.int64), _buf(m + 1, np.int64)
+    lib().ora_compress_rows(A.n_rows, _ptr(A.row_ptr), _ptr(rows), _ptr(rp))
+    return rows[:m], rp
 
 
 def csr5_sigma(A):

@@ -212,6 +212,24 @@ int64_t ora_csr_chunks(int64_t n_rows, const int64_t *row_ptr, int64_t C,
     return k;
 }
 
+/* Compressed rows (A33): the rows of A holding at least one nonzero, in
+ * increasing order, and their row starts followed by nnz -- the CSR of those rows over the
+ * same col/val arrays.  Returns their number. */
+int64_t ora_compress_rows(int64_t n_rows, const int64_t *row_ptr, int64_t *rows_out, int64_t *rp_out)
+{
+    if (n_rows < 0) return -1;
+    int64_t k = 0;
+    for (int64_t r = 0; r < n_rows; ++r) {
+        if (row_ptr[r + 1] > row_ptr[r]) {
+            if (rows_out) rows_out[k] = r;
+            if (rp_out) rp_out[k] = row_ptr[r];
+            ++k;
+        }
+    }
+    if (rp_out) rp_out[k] = n_rows > 0 ? row_ptr[n_rows] : 0;
+    return k;
+}
+
 /* Merge-based CSR: "logically partitions the work ... into equal
  * sized sub-problems".  Work items = n_rows row ends + nnz nonzeros; tile t takes
  * diagonals [t*T, (t+1)*T). */

@@ -84,6 +84,7 @@ int ora_merge_class(int64_t n_rows, const int64_t *row_ptr, int64_t T,
  * ceil(len/C) chunks of C nonzeros (the last one shorter), chunk j of row r starting at
  * row_ptr[r] + j*C; chunks listed by ascending row, then j.  Returns the number of
  * chunks (negative on bad input); chunk_row/chunk_lo (nullable) receive them. */
+int64_t ora_compress_rows(int64_t n_rows, const int64_t *row_ptr, int64_t *rows_out, int64_t *rp_out);
 int64_t ora_csr_chunks(int64_t n_rows, const int64_t *row_ptr, int64_t C,
                        int64_t *chunk_row, int64_t *chunk_lo);
 

@@ -513,4 +513,21 @@ spmv_status spmv_gather(spmv_ctx *ctx, spmv_dtype dtype, const void *src, const 
     return gather_impl(ctx, dtype, src, idx, n, dst, as_stream(stream));
 }
 
+spmv_status spmv_scatter(spmv_ctx *ctx, spmv_dtype dtype, const void *src, const int32_t *idx, int64_t n, void *dst,
+                         void *stream) {
+    if (!ctx || n < 0 || (n > 0 && (!src || !idx || !dst))) { set_error("bad args"); return SPMV_ERR_INVALID_ARG; }
+    if (dtype != SPMV_F32 && dtype != SPMV_F64) { set_error("bad dtype"); return SPMV_ERR_INVALID_ARG; }
+    SPMV_ON_DEVICE(ctx->device);
+    return scatter_impl(ctx, dtype, src, idx, n, dst, as_stream(stream));
+}
+
+spmv_status spmv_compress_rows(spmv_ctx *ctx, const spmv_csr *A, void *stream, int32_t *rows_out, void *rp_out,
+                               int64_t *count_host) {
+    if (!ctx || !count_host || !rp_out || (A && A->n_rows > 0 && !rows_out)) { set_error("bad args"); return SPMV_ERR_INVALID_ARG; }
+    SPMV_TRY(check_csr(A));
+    if (A->n_rows > INT32_MAX) { set_error("compress_rows: more than 2^31 - 1 rows"); return SPMV_ERR_INVALID_ARG; }
+    SPMV_ON_DEVICE(ctx->device);
+    return compress_rows_impl(ctx, A, as_stream(stream), rows_out, rp_out, count_host);
+}
+
 }  // extern "C"

@@ -129,6 +129,10 @@ spmv_status pack_index_impl(spmv_ctx *ctx, const int32_t *colmap, const int64_t 
                             int64_t slot, cudaStream_t s, int32_t *idx, int64_t *count);
 spmv_status gather_impl(spmv_ctx *ctx, spmv_dtype dt, const void *src, const int32_t *idx, int64_t n, void *dst,
                         cudaStream_t s);
+spmv_status scatter_impl(spmv_ctx *ctx, spmv_dtype dt, const void *src, const int32_t *idx, int64_t n, void *dst,
+                         cudaStream_t s);
+spmv_status compress_rows_impl(spmv_ctx *ctx, const spmv_csr *A, cudaStream_t s, int32_t *rows_out, void *rp_out,
+                               int64_t *count);
 spmv_status split_impl(spmv_ctx *ctx, const spmv_csr *A, const int64_t *splits, int nparts, int part,
                        const int32_t *colmap, int which, cudaStream_t s, int32_t *rp_out, int32_t *col_out,
                        void *val_out, int64_t *nnz_out);

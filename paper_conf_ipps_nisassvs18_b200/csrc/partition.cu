@@ -113,6 +113,30 @@ __global__ void k_gather(const V *src, const int *idx, int64_t n, V *dst) {
     for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x)
         dst[q] = src[__ldg(idx + q)];
 }
+template <typename V>
+__global__ void k_scatter(const V *src, const int *idx, int64_t n, V *dst) {
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x)
+        dst[__ldg(idx + q)] = src[q];
+}
+
+// compressed rows (A33): flag[r] = row r has a nonzero; then rows_out[pos[r]] = r and
+// rp_out[pos[r]] = rp[r] for those rows, rp_out[count] = rp[n]
+template <typename IT>
+__global__ void k_nonempty(const IT *rp, int64_t n, int64_t *flag) {
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x)
+        flag[r] = (int64_t)rp[r + 1] > (int64_t)rp[r] ? 1 : 0;
+}
+template <typename IT>
+__global__ void k_compress_rows(const IT *rp, int64_t n, const int64_t *pos, int32_t *rows_out, IT *rp_out) {
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r <= n; r += (int64_t)gridDim.x * blockDim.x) {
+        if (r == n) {
+            rp_out[pos[n]] = rp[n];
+        } else if ((int64_t)rp[r + 1] > (int64_t)rp[r]) {
+            rows_out[pos[r]] = (int32_t)r;
+            rp_out[pos[r]] = rp[r];
+        }
+    }
+}
 
 // own / foreign split of a shard
 template <typename IT>
@@ -298,6 +322,41 @@ spmv_status gather_impl(spmv_ctx *ctx, spmv_dtype dt, const void *src, const int
     else k_gather<float><<<blocks_for(ctx, n), 256, 0, s>>>((const float *)src, idx, n, (float *)dst);
     SPMV_LAUNCH_CHECK();
     return SPMV_OK;
+}
+
+spmv_status scatter_impl(spmv_ctx *ctx, spmv_dtype dt, const void *src, const int32_t *idx, int64_t n, void *dst,
+                         cudaStream_t s) {
+    if (n <= 0) return SPMV_OK;
+    if (dt == SPMV_F64) k_scatter<double><<<blocks_for(ctx, n), 256, 0, s>>>((const double *)src, idx, n, (double *)dst);
+    else k_scatter<float><<<blocks_for(ctx, n), 256, 0, s>>>((const float *)src, idx, n, (float *)dst);
+    SPMV_LAUNCH_CHECK();
+    return SPMV_OK;
+}
+
+template <typename IT>
+spmv_status compress_rows_t(spmv_ctx *ctx, const spmv_csr *A, cudaStream_t s, int32_t *rows_out, void *rp_out,
+                            int64_t *count) {
+    const int64_t n = A->n_rows;
+    const IT *rp = (const IT *)A->row_ptr;
+    Scratch flag(ctx, s), pos(ctx, s);
+    SPMV_TRY(flag.alloc(std::max<int64_t>(n, 1) * 8));
+    SPMV_TRY(pos.alloc((n + 1) * 8));
+    if (n) {
+        k_nonempty<IT><<<blocks_for(ctx, n), 256, 0, s>>>(rp, n, flag.as<int64_t>());
+        SPMV_LAUNCH_CHECK();
+    }
+    SPMV_TRY(exclusive_scan_i64(ctx, flag.as<int64_t>(), pos.as<int64_t>(), n, s));
+    k_compress_rows<IT><<<blocks_for(ctx, n + 1), 256, 0, s>>>(rp, n, pos.as<int64_t>(), rows_out, (IT *)rp_out);
+    SPMV_LAUNCH_CHECK();
+    SPMV_CUDA_TRY(cudaMemcpyAsync(count, pos.as<int64_t>() + n, 8, cudaMemcpyDeviceToHost, s));
+    SPMV_CUDA_TRY(cudaStreamSynchronize(s));
+    return SPMV_OK;
+}
+
+spmv_status compress_rows_impl(spmv_ctx *ctx, const spmv_csr *A, cudaStream_t s, int32_t *rows_out, void *rp_out,
+                               int64_t *count) {
+    if (A->ptr_type == SPMV_I32) return compress_rows_t<int>(ctx, A, s, rows_out, rp_out, count);
+    return compress_rows_t<int64_t>(ctx, A, s, rows_out, rp_out, count);
 }
 
 template <typename IT, typename V>

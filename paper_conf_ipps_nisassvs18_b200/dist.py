@@ -31,7 +31,7 @@ import numpy as np
 import torch
 import torch.distributed as dist
 
-from .spmv import (CSR, convert, partition, slice_remap, spmv_colmap_pack_index, spmv_gather, spmv_halo_colmap,
+from .spmv import (CSR, convert, partition, slice_remap, spmv_colmap_pack_index, spmv_compress_rows, spmv_gather, spmv_halo_colmap, spmv_scatter,
                    spmv_partition_colmap, spmv_slice_remap_colmap, spmv_slice_split)
 
 
@@ -346,14 +346,45 @@ class HaloPlan:
         return all_to_all_slots(recv_buf, send_buf, [self.S] * self.P, self.slots, group=group, async_op=async_op)
 
 
+def _compressed_faster(full, comp, rows, yf, n_rows, n_cols, reps: int = 5) -> bool:
+    """A33 choice on this rank: the foreign block over every row (one run) or over its
+    non-empty rows (gather, run, scatter) -- whichever takes less device time (CUDA events
+    around `reps` back-to-back steps, after a warm-up; scratch vectors)."""
+    dt = yf.dtype
+    y = torch.zeros(n_rows, dtype=dt, device=yf.device)
+    x = torch.zeros(max(n_cols, 1), dtype=dt, device=yf.device)
+    s = torch.cuda.current_stream()
+
+    def t(fn):
+        fn()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(s)
+        for _ in range(reps):
+            fn()
+        b.record(s)
+        b.synchronize()
+        return a.elapsed_time(b)
+
+    def run_comp():
+        spmv_gather(y, rows, yf)
+        comp.run(1.0, x, 1.0, yf)
+        spmv_scatter(yf, rows, y)
+
+    return t(run_comp) < t(lambda: full.run(1.0, x, 1.0, y))
+
+
 class HaloSpMV:
     """Row-partitioned y = alpha*A*x + beta*y with a halo exchange instead of the x
     all-gather.  Own-column block on the rank's x slice (overlapping
     the exchange on NCCL), foreign-column block on the received halo (beta = 1)."""
 
-    def __init__(self, A: CSR, fmt: str = "csr", group=None, **convert_opts):
+    def __init__(self, A: CSR, fmt: str = "csr", group=None, foreign: str = "auto", **convert_opts):
+        """foreign: "auto" (A33: the faster of the two on this rank), "full" (the foreign
+        block over every row) or "compressed" (over its non-empty rows)."""
         if A.n_rows != A.n_cols:
             raise ValueError("HaloSpMV needs a square matrix (x is owned like y)")
+        if foreign not in ("auto", "full", "compressed"):
+            raise ValueError(foreign)
         self.group = group
         P = dist.get_world_size(group)
         rank = dist.get_rank(group)
@@ -363,9 +394,22 @@ class HaloSpMV:
         self.fmt = fmt
         self.plan = HaloPlan(A, splits, rank)
         self.own = convert(spmv_slice_split(A, splits, rank, 0), fmt, **convert_opts)
-        self.foreign = convert(spmv_slice_split(A, splits, rank, 1, self.plan.colmap, self.plan.S), fmt,
-                               **convert_opts)
+        F = spmv_slice_split(A, splits, rank, 1, self.plan.colmap, self.plan.S)
+        # A33: a banded matrix's foreign block holds a few thousand non-empty rows among the
+        # rank's millions -- run it over those rows only (gather their y, SpMV with beta = 1,
+        # scatter back: the same single rounding as the full block), not over every row --
+        # when that is faster for this format and shard: the formats that walk every row
+        # (CSR, ELL/HYB, merge) gain on large shards, the nonzero-driven ones (COO, CSR5)
+        # already skip rows without work and lose the extra launches (tools/halo_local_time.py)
         dev, self.dtype = A.row_ptr.device, A.val.dtype
+        rows, rp_c = spmv_compress_rows(F)
+        self.frows, self.yf = None, torch.zeros(0, dtype=self.dtype, device=dev)
+        self.foreign = convert(F, fmt, **convert_opts) if F.nnz > 0 else None
+        if self.foreign is not None and foreign != "full" and (foreign == "compressed" or rows.numel() * 4 <= F.n_rows):
+            comp = convert(CSR(rp_c, F.col, F.val, (rows.numel(), F.n_cols)), fmt, **convert_opts)
+            yf = torch.zeros(rows.numel(), dtype=self.dtype, device=dev)
+            if foreign == "compressed" or _compressed_faster(self.foreign, comp, rows, yf, F.n_rows, F.n_cols):
+                self.foreign, self.frows, self.yf = comp, rows, yf
         self.x_own = torch.zeros(self.layout.rows, dtype=self.dtype, device=dev)
         self.send = torch.zeros(self.plan.send_index.numel(), dtype=self.dtype, device=dev)
         self.recv = torch.zeros(self.plan.recv_len, dtype=self.dtype, device=dev)
@@ -393,20 +437,37 @@ class HaloSpMV:
         self.own.run(alpha, self.x_own, beta, y_local)              # overlaps the exchange
         if work is not None:
             work.wait()
-        self.foreign.run(alpha, self.recv, 1.0, y_local)
+        self._foreign(alpha, y_local)
         return y_local
+
+    def _foreign(self, alpha, y_local: torch.Tensor):
+        if self.foreign is None:
+            return
+        if self.frows is None:
+            self.foreign.run(alpha, self.recv, 1.0, y_local)
+        elif self.frows.numel():
+            spmv_gather(y_local, self.frows, self.yf)
+            self.foreign.run(alpha, self.recv, 1.0, self.yf)
+            spmv_scatter(self.yf, self.frows, y_local)
 
     def run_local(self, alpha, beta, y_local: torch.Tensor):
         self.own.run(alpha, self.x_own, beta, y_local)
-        self.foreign.run(alpha, self.recv, 1.0, y_local)
+        self._foreign(alpha, y_local)
         return y_local
 
     def local_bytes(self) -> int:
-        return self.own.info()["bytes_per_run"] + self.foreign.info()["bytes_per_run"] - \
-            self.rows * self.x_own.element_size() * 2
+        V = self.x_own.element_size()
+        b = self.own.info()["bytes_per_run"]
+        if self.foreign is None:
+            return b
+        if self.frows is None:                  # y read + written once, by the own block
+            return b + self.foreign.info()["bytes_per_run"] - self.rows * V * 2
+        k = self.frows.numel()                  # + gather / scatter of the compressed rows' y
+        return b + self.foreign.info()["bytes_per_run"] + k * (4 + V) * 2
 
     def launches(self) -> int:
-        return self.own.launches() + self.foreign.launches() + 1
+        f = 0 if self.foreign is None else self.foreign.launches() + (2 if self.frows is not None else 0)
+        return self.own.launches() + f + 1
 
     def gather_y(self, y_local: torch.Tensor) -> torch.Tensor:
         P, S = self.layout.P, self.layout.S

@@ -137,6 +137,8 @@ def lib():
             "spmv_colmap_pack_index": (C.c_int, [_P, _P, C.POINTER(C.c_int64), C.c_int, C.c_int, C.c_int64, _P, _P,
                                                  C.POINTER(C.c_int64)]),
             "spmv_gather": (C.c_int, [_P, C.c_int, _P, _P, C.c_int64, _P, _P]),
+            "spmv_scatter": (C.c_int, [_P, C.c_int, _P, _P, C.c_int64, _P, _P]),
+            "spmv_compress_rows": (C.c_int, [_P, C.POINTER(spmv_csr), _P, _P, _P, C.POINTER(C.c_int64)]),
             "spmv_halo_colmap": (C.c_int, [_P, C.POINTER(spmv_csr), C.POINTER(C.c_int64), C.c_int, C.c_int, _P, _P,
                                            C.POINTER(C.c_int64), C.POINTER(C.c_int64)]),
             "spmv_slice_split": (C.c_int, [_P, C.POINTER(spmv_csr), C.POINTER(C.c_int64), C.c_int, C.c_int, _P,
@@ -445,6 +447,33 @@ def spmv_gather(src: torch.Tensor, idx: torch.Tensor, dst: torch.Tensor, stream=
                              idx.data_ptr() if n else None, n, dst.data_ptr() if dst.numel() else None,
                              _stream_ptr(stream)))
     return dst
+
+
+def spmv_scatter(src: torch.Tensor, idx: torch.Tensor, dst: torch.Tensor, stream=None):
+    """dst[idx[q]] = src[q] on the GPU (idx distinct; the inverse of spmv_gather, A33)."""
+    ctx = context(src.device.index)
+    n = idx.numel()
+    dt = 1 if src.dtype == torch.float64 else 0
+    _check(lib().spmv_scatter(ctx.ptr, dt, src.data_ptr() if src.numel() else None,
+                              idx.data_ptr() if n else None, n, dst.data_ptr() if dst.numel() else None,
+                              _stream_ptr(stream)))
+    return dst
+
+
+def spmv_compress_rows(A: CSR, stream=None):
+    """A's non-empty rows (int32 [count]) and their row starts followed by nnz ([count + 1],
+    A's index type): (rows, rp) with CSR(rp, A.col, A.val) the compressed-row block (A33)."""
+    ctx = context(A.row_ptr.device.index)
+    n = A.n_rows
+    dev = A.row_ptr.device
+    rows = torch.empty(max(n, 1), dtype=torch.int32, device=dev)
+    rp = torch.empty(n + 1, dtype=A.row_ptr.dtype, device=dev)
+    cnt = C.c_int64()
+    a = A.as_c()
+    _check(lib().spmv_compress_rows(ctx.ptr, C.byref(a), _stream_ptr(stream), rows.data_ptr(), rp.data_ptr(),
+                                    C.byref(cnt)))
+    k = cnt.value
+    return rows[:k], rp[:k + 1]
 
 
 # ----------------------------------------------------------------- handle

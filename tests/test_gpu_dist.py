@@ -280,3 +280,40 @@ def test_halo_colmap_bit_exact(sp, case, P):
         for snd in range(P):
             idx = spmv_colmap_pack_index(cm, splits, snd, S).cpu().numpy()
             assert np.array_equal(idx, oracle.halo_pack_index(cmo, splits, snd, So)), (k, snd)
+
+
+@pytest.mark.parametrize("ptr", [torch.int32, torch.int64], ids=["i32", "i64"])
+@pytest.mark.parametrize("case", ["sparse_rows", "no_empty", "all_empty", "lap_foreign"])
+def test_compress_rows_bit_exact(sp, case, ptr):
+    """spmv_compress_rows (A33) equals the oracle's compressed rows bit for bit, and
+    spmv_scatter puts a gathered vector back (dst[idx[q]] = src[q])."""
+    from paper_conf_ipps_nisassvs18_b200.dist import HaloPlan
+    from paper_conf_ipps_nisassvs18_b200.spmv import partition, spmv_compress_rows, spmv_gather, spmv_scatter, spmv_slice_split
+    rng = np.random.default_rng(41)
+    if case == "lap_foreign":                       # a rank's foreign block of a 4-way Laplacian split
+        dA = sp.CSR.from_host(matgen.laplacian5(96))
+        splits = partition(dA, 4)
+        plan = HaloPlan(dA, splits, 1)
+        F = spmv_slice_split(dA, splits, 1, 1, plan.colmap, plan.S)
+        A = matgen.HostCSR(F.row_ptr.cpu().numpy().astype(np.int64), F.col.cpu().numpy(), F.val.cpu().numpy(),
+                           F.n_rows, F.n_cols)
+    else:
+        lens = {"sparse_rows": np.where(rng.random(70000) < 0.01, rng.integers(1, 9, 70000), 0),
+                "no_empty": rng.integers(1, 5, 3000), "all_empty": np.zeros(5000, np.int64)}[case]
+        A = matgen.from_lengths(lens, 4000, seed=42)
+    dA = sp.CSR.from_host(A, ptr_dtype=ptr)
+    rows, rp = spmv_compress_rows(dA)
+    orows, orp = oracle.compress_rows(A)
+    assert rows.dtype == torch.int32 and rp.dtype == ptr
+    assert np.array_equal(rows.cpu().numpy().astype(np.int64), orows)
+    assert np.array_equal(rp.cpu().numpy().astype(np.int64), orp)
+    y = torch.from_numpy(matgen.vector(A.n_rows, 43, 1)).cuda()
+    yc = torch.empty(rows.numel(), dtype=torch.float64, device="cuda")
+    spmv_gather(y, rows, yc)
+    z = torch.zeros_like(y)
+    spmv_scatter(yc, rows, z)
+    torch.cuda.synchronize()
+    keep = np.zeros(A.n_rows, bool)
+    keep[orows] = True
+    assert np.array_equal(z.cpu().numpy()[keep], y.cpu().numpy()[keep])
+    assert not z.cpu().numpy()[~keep].any()

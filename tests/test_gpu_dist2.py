@@ -74,10 +74,14 @@ def _worker(rank, world, port, q):
         A = matgen.laplacian5(64, kind="int")
         x = matgen.vector(A.n_cols, 55, 1, "int")
         y = matgen.vector(A.n_rows, 55, 2, "int")
-        for fmt in ("csr", "ell", "csr5"):
-            op = HaloSpMV(sp.CSR.from_host(A), fmt)
-            ok, how = _check(step(op, A, x, y, 2.0, -1.0), A, x, y, 2.0, -1.0, True)
-            out.append((f"halo lap64 {fmt} S={op.plan.S}", ok and op.plan.S <= 64, how))
+        for fmt in ("csr", "ell", "csr5", "coo", "hyb", "merge"):
+            for foreign in ("full", "compressed", "auto"):
+                op = HaloSpMV(sp.CSR.from_host(A), fmt, foreign=foreign)
+                ok, how = _check(step(op, A, x, y, 2.0, -1.0), A, x, y, 2.0, -1.0, True)
+                # compressed: the foreign block runs over its 64 boundary rows only (A33)
+                shape = (op.frows is None) if foreign == "full" else \
+                    (op.frows is not None and op.frows.numel() == 64) if foreign == "compressed" else True
+                out.append((f"halo lap64 {fmt} S={op.plan.S} foreign={foreign}", ok and op.plan.S <= 64 and shape, how))
         # rank-local R-MAT: GPU generator, values of the rank's rows only
         for kind, exact in (("int", True), ("f64", False)):
             Ah = matgen.rmat(12, seed=56, kind=kind)

@@ -574,3 +574,36 @@ def test_oracle_hot_columns_brute_force(case, kmax):
     if hot.size:
         rest = deg[(deg > 0) & (deg < t)]
         assert rest.size == 0 or rest.max() < deg[hot].min()
+
+
+# ---- A33: compressed rows (the foreign-column block of a halo step)
+
+def test_compress_rows_hand_example():
+    # rows 0..4 of lengths 0, 2, 0, 1, 0: the non-empty rows are 1 and 3
+    A = matgen.HostCSR(np.array([0, 0, 2, 2, 3, 3], np.int64), np.array([1, 4, 0], np.int32), np.ones(3), 5, 5)
+    rows, rp = oracle.compress_rows(A)
+    assert rows.tolist() == [1, 3] and rp.tolist() == [0, 2, 3]
+
+
+@pytest.mark.parametrize("case", ["no_empty", "all_empty", "zero_rows", "sparse_rows"])
+def test_compress_rows_special_cases_and_round_trip(case):
+    """No empty row: the identity (rows = 0..n-1, rp unchanged); all rows empty: nothing
+    and rp = [0]; n = 0: nothing; otherwise expanding (rows, rp) back over all rows
+    reproduces row_ptr, so the compressed CSR holds exactly A's nonzeros, row by row."""
+    rng = np.random.default_rng(33)
+    lens = {"no_empty": rng.integers(1, 9, 500), "all_empty": np.zeros(300, np.int64),
+            "zero_rows": np.zeros(0, np.int64),
+            "sparse_rows": np.where(rng.random(5000) < 0.02, rng.integers(1, 7, 5000), 0)}[case]
+    A = matgen.from_lengths(lens, 1000, seed=5)
+    rows, rp = oracle.compress_rows(A)
+    n = A.n_rows
+    if case == "no_empty":
+        assert np.array_equal(rows, np.arange(n)) and np.array_equal(rp, A.row_ptr)
+    if case in ("all_empty", "zero_rows"):
+        assert rows.size == 0 and rp.tolist() == [0]
+    assert np.all(np.diff(rows) > 0) and np.all(np.diff(rp) > 0)
+    back = np.zeros(n + 1, np.int64)                  # expand: row r ends where its successor starts
+    full = np.zeros(n, np.int64)
+    full[rows] = np.diff(rp)
+    np.cumsum(full, out=back[1:])
+    assert np.array_equal(back, A.row_ptr)
