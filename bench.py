@@ -46,6 +46,9 @@ CONFIGS = {
     "rmat24": dict(desc="BASELINE configs[2]: R-MAT scale 24, edge factor 16, Graph500 (a,b,c)=(.57,.19,.19)"),
     "rmat27": dict(desc="BASELINE configs[4]: R-MAT scale 27, edge factor 16, Graph500 (a,b,c)=(.57,.19,.19), "
                         "int64 row_ptr"),
+    "rgg19": dict(desc="synthetic stand-in for rgg_n_2_19_s0 (the matrix PAPER.md:131 quotes): random geometric "
+                       "graph, 2^19 points in the unit square, r = 0.55 sqrt(ln n / n), grid-cell numbering "
+                       "(matgen.rgg; 524,288 rows, 6.55M nnz vs the file's 6.54M)"),
 }
 RMAT_FORMATS = {"rmat24": "coo,csr,hyb,merge,csr5", "rmat27": "csr,merge,csr5"}
 
@@ -81,6 +84,8 @@ def build_matrix(name, dtype_kind):
         return matgen.laplacian5(int(name[3:]))
     if name.startswith("rmat"):
         return matgen.rmat(int(name[4:]), seed=matgen.SEEDS.get(name, matgen.SEEDS["rmat24"]), kind=dtype_kind)
+    if name.startswith("rgg"):
+        return matgen.rgg(int(name[3:]), seed=matgen.SEEDS.get(name, matgen.SEEDS["rgg19"]), kind=dtype_kind)
     if name.startswith("mtx:"):                     # a Matrix Market file
         from matgen.mtx import read_mtx
         A = read_mtx(name[4:])
@@ -516,15 +521,16 @@ def consistency(handles, x, y_init, dtype):
     return ok, agree
 
 
-def extra_rmat24(sp, args, peak, peak_src, local):
-    """configs[2] (R-MAT 24) per-format blocks in fp64 and fp32 beside the headline."""
+def extra_rmat24(sp, args, peak, peak_src, local, config="rmat24", formats=None):
+    """configs[2] (R-MAT 24) per-format blocks in fp64 and fp32 beside the headline (and the
+    same for the rgg19 stand-in of the paper's rgg_n_2_19_s0)."""
     import torch
 
     from matgen import gpu
     out = {}
     stream = torch.cuda.current_stream()
     for dname, dtype, kind in (("f64", torch.float64, "f64"), ("f32", torch.float32, "f32")):
-        dA, _ = device_matrix("rmat24", kind, dtype)
+        dA, _ = device_matrix(config, kind, dtype)
         feats = sp.features(dA)
         torch.cuda.synchronize()
         ft = []
@@ -534,16 +540,16 @@ def extra_rmat24(sp, args, peak, peak_src, local):
             ft.append(time.perf_counter() - t0)
         ft.sort()
         fbytes = (dA.n_rows + 1) * dA.row_ptr.element_size() + 4 * dA.nnz
-        handles, conv_ms, na = convert_all(sp, dA, RMAT_FORMATS["rmat24"].split(","), feats)
+        handles, conv_ms, na = convert_all(sp, dA, (formats or RMAT_FORMATS["rmat24"]).split(","), feats)
         x = gpu.vector(dA.n_cols, 0x5EED0003, 1, kind, dtype)
         y0 = gpu.vector(dA.n_rows, 0x5EED0003, 2, kind, dtype)
         ok, agree = consistency(handles, x, y0, dtype)
         if not ok:
-            raise SystemExit(f"rmat24 {dname}: formats disagree {agree}")
+            raise SystemExit(f"{config} {dname}: formats disagree {agree}")
         steps = max(5, min(args.steps, args.extra_steps))
         ms_step, per, clocks, variants = time_formats(handles, x, y0, steps, args.warmup, local, stream,
                                                       extra_variants=False)
-        pf = format_block(handles, per, {}, dA.nnz, peak, "rmat24", dname, conv_ms)
+        pf = format_block(handles, per, {}, dA.nnz, peak, config, dname, conv_ms)
         for f, why in na.items():
             pf[f] = {"status": "N/A", "reason": why}
         fm = [f for f in handles]
@@ -705,6 +711,15 @@ def run_single(args):
         handles = None
         torch.cuda.empty_cache()
         extra = {"rmat24": extra_rmat24(sp, args, peak, peak_src, 0)}
+        rg = extra_rmat24(sp, args, peak, peak_src, 0, config="rgg19", formats=",".join(sp.PAPER_FORMATS))
+        # R1: the paper's own numbers for this matrix (K80c, single precision, the real file)
+        # beside ours (B200, the synthetic stand-in, fp32 storage with fp64 accumulation)
+        rg["vs_paper"] = {f: {"paper_k80c_gflops": g, "b200_gflops_f32": rg["f32"]["per_format"][f]["gflops"]}
+                          for f, g in (("csr5", 22), ("merge", 21)) if "gflops" in rg["f32"]["per_format"].get(f, {})}
+        rg["vs_paper"]["source"] = "PAPER.md:131 (rgg_n_2_19_s0 on a Tesla K80c)"
+        rg["l2"] = ("the matrix (~80 MB in fp64) fits the 126 MB L2: back-to-back runs are L2-warm, as in the "
+                    "paper's timing loop (A11); frac_of_peak is against HBM and can overstate")
+        extra["rgg19"] = rg
 
     line = {
         "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": 1, "steps": args.steps,

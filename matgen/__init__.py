@@ -20,7 +20,7 @@ _LIB_PATH = os.path.join(_HERE, "libmatgen.so")
 VALUE_KINDS = {"f64": 0, "f32": 1, "int": 2, "ones": 3}
 
 SEEDS = {"u2048": 0x5EED0001, "lap4096": 0x5EED0002, "rmat24": 0x5EED0003,
-         "sweep": 0x5EED1000, "rmat27": 0x5EED0005}
+         "sweep": 0x5EED1000, "rmat27": 0x5EED0005, "rgg19": 0x5EED0019}
 
 
 def build(force: bool = False) -> str:
@@ -162,6 +162,51 @@ def rmat(scale, edge_factor=16, seed=SEEDS["rmat24"], abc=(0.57, 0.19, 0.19), ki
     lib().mg_keys_to_csr(_ptr(keys), int(m), int(scale), int(n), _ptr(row_ptr), _ptr(col))
     del keys
     A = HostCSR(row_ptr, col, np.empty(0), n, n, f"rmat{scale}")
+    return set_values(A, seed + 11, kind)
+
+
+def rgg(scale, seed=SEEDS["rgg19"], kind="f64", r_coef=0.55) -> HostCSR:
+    """Random geometric graph by the recipe of DIMACS10 rgg_n_2_{scale}_s0 (SuiteSparse;
+    the matrix PAPER.md:131 quotes CSR5 / merge GFLOP/s on): n = 2^scale points uniform in
+    the unit square, an edge between two distinct points closer than r = r_coef*sqrt(ln n/n)
+    (symmetric pattern, no self loops); points numbered in grid-cell order (cells of side
+    >= r, row-major; by x inside a cell), so neighbours get nearby indices.  A synthetic
+    stand-in -- the SuiteSparse file is not reachable here -- with the same size and degree
+    law (scale 19: 524,288 rows; rgg_n_2_19_s0 has 6,539,532 nonzeros).  Values
+    position-keyed (A18)."""
+    n = 1 << int(scale)
+    rng = np.random.default_rng(seed)
+    pts = rng.random((n, 2))
+    r = r_coef * np.sqrt(np.log(n) / n)
+    nc = max(1, int(1.0 / r))                              # cells per side, side 1/nc >= r
+    cxy = np.minimum((pts * nc).astype(np.int64), nc - 1)
+    cell = cxy[:, 1] * nc + cxy[:, 0]
+    order = np.lexsort((pts[:, 0], cell))
+    pts, cell, cxy = pts[order], cell[order], cxy[order]
+    starts = np.searchsorted(cell, np.arange(nc * nc + 1))
+    ii, jj = [], []
+    idx = np.arange(n, dtype=np.int64)
+    for dy in (-1, 0, 1):
+        for dx in (-1, 0, 1):
+            ny, nx = cxy[:, 1] + dy, cxy[:, 0] + dx
+            ok = (ny >= 0) & (ny < nc) & (nx >= 0) & (nx < nc)
+            c2 = np.where(ok, ny * nc + nx, 0)
+            lo = starts[c2]
+            cnt = np.where(ok, starts[c2 + 1] - lo, 0)
+            tot = int(cnt.sum())
+            i = np.repeat(idx, cnt)
+            j = np.repeat(lo, cnt) + (np.arange(tot, dtype=np.int64) - np.repeat(np.cumsum(cnt) - cnt, cnt))
+            d = pts[i] - pts[j]
+            keep = (i != j) & ((d * d).sum(axis=1) < r * r)
+            ii.append(i[keep])
+            jj.append(j[keep])
+    i = np.concatenate(ii)
+    j = np.concatenate(jj)
+    o = np.lexsort((j, i))
+    i, j = i[o], j[o]
+    row_ptr = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(np.bincount(i, minlength=n), out=row_ptr[1:])
+    A = HostCSR(row_ptr, j.astype(np.int32), np.empty(0), n, n, f"rgg{scale}")
     return set_values(A, seed + 11, kind)
 
 

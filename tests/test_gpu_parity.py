@@ -58,6 +58,7 @@ def edge_cases(kind="f64"):
     cases["lap64"] = matgen.laplacian5(64, kind=kind)
     cases["rmat12"] = matgen.rmat(12, seed=12, kind=kind)
     cases["rmat15"] = matgen.rmat(15, seed=15, kind=kind)
+    cases["rgg12"] = matgen.rgg(12, seed=12, kind=kind)      # the paper's rgg_n_2_k_s0 recipe
     cases["banded"] = matgen.window(3000, 3000, 9, 0.6, seed=9, mode=0, kind=kind)
     cases["blockdiag"] = matgen.window(2500, 4000, 64, 0.8, seed=10, mode=1, kind=kind)
     cases["poisson_rect"] = _lens_matrix(rng.poisson(20, 4000), 1500, 11, kind)
@@ -85,7 +86,7 @@ def case(name, kind):
 
 
 CASE_NAMES = ["empty0x0", "1x1", "dense_row_1x5000", "col_n_x_1", "rect_3x7", "rect_7x3", "nnz0_rows5",
-              "empty_runs", "long_row", "tile_bounds", "u2048", "lap37", "lap64", "rmat12", "rmat15",
+              "empty_runs", "long_row", "tile_bounds", "u2048", "lap37", "lap64", "rmat12", "rmat15", "rgg12",
               "banded", "blockdiag", "poisson_rect", "all_zero_vals", "sparse_rows", "mixed_sparse"]
 
 
