@@ -130,3 +130,30 @@ def test_full_size_rmat27_sampled(sp):
         del dA, val
         torch.cuda.empty_cache()
     g.release()
+
+
+@pytest.mark.parametrize("seed", [101, 202, 303])
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32], ids=["f64", "f32"])
+def test_dynamic_csr_random_shapes(sp, seed, dtype):
+    """Randomized shapes at the CSR-vector dynamic-scheduling size (2M rows): a mix of empty
+    runs, short rows, rows just over the group width, 40..300-long rows and rows past the
+    chunk threshold (A25), in random order -- CSR (and CSR5 / merge on the same matrix)
+    within the bound on every row, beta = 0.75."""
+    rng = np.random.default_rng(seed)
+    n = 2_000_000
+    kind = rng.choice(5, size=n, p=[0.45, 0.35, 0.12, 0.0795, 0.0005])
+    lens = np.select([kind == 0, kind == 1, kind == 2, kind == 3, kind == 4],
+                     [0, rng.integers(1, 17, n), rng.integers(17, 40, n), rng.integers(40, 301, n),
+                      rng.integers(1025, 20000, n)])
+    k = "f64" if dtype == torch.float64 else "f32"
+    A = matgen.from_lengths(lens, 3_000_000, seed=seed, kind=k)
+    dA = sp.CSR.from_host(A, dtype=dtype)
+    x = matgen.vector(A.n_cols, seed, 1, k)
+    y = matgen.vector(A.n_rows, seed, 2, k)
+    ref, bound = oracle.spmv_csr(A, x, 1.25, 0.75, y, with_bound=True)
+    xd = torch.from_numpy(x).cuda().to(dtype)
+    yd0 = torch.from_numpy(y).cuda().to(dtype)
+    for fmt in ("csr", "csr5", "merge"):
+        out = _run(sp, dA, fmt, 1.25, xd, 0.75, yd0).cpu().double().numpy()
+        ok, ratio, nbad = oracle.check_tolerance(out, ref, bound, 1e-12 if dtype == torch.float64 else 1e-5)
+        assert ok, (fmt, nbad, ratio)
