@@ -107,129 +107,129 @@ k_csr_vector(const IT *__restrict__ rp, const int *__restrict__ col, const V *__
     // lane (sub < U) of each row writes y[my_row] (row_ok)
     auto batch = [&](const IT (&a)[U], const IT (&b)[U], const IT ra0, const IT rhi, const bool contiguous,
                      const bool slot_ok, const int64_t my_row, const bool row_ok) {
-            // the y value this lane will write (writer lane sub == u of group g)
-            const double yv = (!B0 && sub < U && row_ok) ? (double)y[my_row] : 0.0;
-            // first W elements of every row, all loads issued together
-            int c0[U];
-            V v0[U];
-    #pragma unroll
-            for (int u = 0; u < U; ++u) {
-                const int64_t k = (int64_t)a[u] + sub;
-                c0[u] = k < b[u] ? ld_hint(col + k, pa) : -1;
-                v0[u] = k < b[u] ? ld_hint(val + k, pa) : (V)0;
+        // the y value this lane will write (writer lane sub == u of group g)
+        const double yv = (!B0 && sub < U && row_ok) ? (double)y[my_row] : 0.0;
+        // first W elements of every row, all loads issued together
+        int c0[U];
+        V v0[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t k = (int64_t)a[u] + sub;
+            c0[u] = k < b[u] ? ld_hint(col + k, pa) : -1;
+            v0[u] = k < b[u] ? ld_hint(val + k, pa) : (V)0;
+        }
+        double s[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) s[u] = c0[u] != -1 ? (double)v0[u] * (double)ldx<HOT>(x, xh, c0[u], px) : 0.0;
+        // the group's U results: lane sub == u of group g writes row u*G + g
+        double mine = 0.0;
+        {
+            // lane bits >= U do not index rows: plain butterflies over them; then a
+            // transpose reduction over the low bits -- at offset o a lane keeps the half
+            // of its partial sums selected by (sub & o) and adds the other half received
+            // from lane sub ^ o, so lane sub ends with row (sub mod U)'s sum (U - 1
+            // shuffles instead of a butterfly per row, U * log2(U))
+#pragma unroll
+            for (int o = W / 2; o >= U; o >>= 1) {
+#pragma unroll
+                for (int u = 0; u < U; ++u) s[u] += __shfl_xor_sync(0xffffffffu, s[u], o);
             }
-            double s[U];
-    #pragma unroll
-            for (int u = 0; u < U; ++u) s[u] = c0[u] != -1 ? (double)v0[u] * (double)ldx<HOT>(x, xh, c0[u], px) : 0.0;
-            // the group's U results: lane sub == u of group g writes row u*G + g
-            double mine = 0.0;
-            {
-                // lane bits >= U do not index rows: plain butterflies over them; then a
-                // transpose reduction over the low bits -- at offset o a lane keeps the half
-                // of its partial sums selected by (sub & o) and adds the other half received
-                // from lane sub ^ o, so lane sub ends with row (sub mod U)'s sum (U - 1
-                // shuffles instead of a butterfly per row, U * log2(U))
-    #pragma unroll
-                for (int o = W / 2; o >= U; o >>= 1) {
-    #pragma unroll
-                    for (int u = 0; u < U; ++u) s[u] += __shfl_xor_sync(0xffffffffu, s[u], o);
+#pragma unroll
+            for (int o = U / 2; o > 0; o >>= 1) {
+                const bool hi = (sub & o) != 0;
+#pragma unroll
+                for (int j = 0; j < o; ++j) {
+                    const double send = hi ? s[j] : s[j + o];
+                    const double keep = hi ? s[j + o] : s[j];
+                    s[j] = keep + __shfl_xor_sync(0xffffffffu, send, o);
                 }
-    #pragma unroll
-                for (int o = U / 2; o > 0; o >>= 1) {
-                    const bool hi = (sub & o) != 0;
-    #pragma unroll
-                    for (int j = 0; j < o; ++j) {
-                        const double send = hi ? s[j] : s[j + o];
-                        const double keep = hi ? s[j + o] : s[j];
-                        s[j] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+            }
+            mine = s[0];
+        }
+        // rows longer than W: the remainder is processed by the WHOLE warp, one row at a
+        // time (the paper's warp-per-row vector kernel), 8 loads per lane in
+        // flight, accumulators folded every kFold steps (A13); lane i holds row i's range
+        {
+            // lane i's row range, derived only here: contiguous batches hold row starts
+            // (the batch end in rhi), compacted ones hold [start, end) directly
+            const IT my_a = ra0;
+            const IT nx = __shfl_sync(0xffffffffu, ra0, (lane + 1) & 31);
+            const IT my_e = contiguous ? (lane + 1 < R ? nx : rhi) : rhi;
+            const int64_t my_len = (int64_t)my_e - (int64_t)my_a;
+            const bool is_long = slot_ok && my_len > W && (!CHUNKED || my_len <= long_len);
+            // remainders of at most kSubMax: all such rows of the batch at once, a subgroup
+            // of SW = 32 / next_pow2(count) lanes per row, 8 predicated loads per lane per
+            // step -- one gather round trip for the batch instead of one per row (R-MAT's
+            // many rows a little longer than W)
+            const unsigned few = __ballot_sync(0xffffffffu, is_long && my_len - W <= kSubMax);
+            unsigned more = __ballot_sync(0xffffffffu, is_long) & ~few;
+            if (few) {
+                const int nl = __popc(few);
+                const int lg = nl > 1 ? 32 - __clz(nl - 1) : 0;
+                const int SW = 32 >> lg;
+                const int sg = lane >> (5 - lg), sl = lane & (SW - 1);
+                const int ri = sg < nl ? (int)__fns(few, 0, sg + 1) : 0;
+                const int64_t ra = (int64_t)__shfl_sync(0xffffffffu, my_a, ri) + W;
+                const int64_t re = (int64_t)__shfl_sync(0xffffffffu, my_e, ri);
+                const int64_t rb = sg < nl ? re : ra;
+                double acc[8];
+#pragma unroll
+                for (int q = 0; q < 8; ++q) acc[q] = 0.0;
+                for (int64_t k = ra + sl; k < rb; k += 8 * SW) {
+                    int d[8];
+                    V w[8];
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) {
+                        const bool in = k + q * SW < rb;
+                        d[q] = in ? ld_hint(col + k + q * SW, pa) : -1;
+                        w[q] = in ? ld_hint(val + k + q * SW, pa) : (V)0;
+                    }
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) if (d[q] != -1) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
+                }
+                double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
+                for (int o = SW >> 1; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+                const int wi = g * U + (sub < U ? sub : 0);           // this lane's row (writer lanes)
+                const bool wmine = sub < U && ((few >> wi) & 1u);
+                const int src = (__popc(few & ((1u << wi) - 1u)) << (5 - lg)) & 31;
+                const double got = __shfl_sync(0xffffffffu, part, src);
+                if (wmine) mine += got;
+            }
+            while (more) {
+                const int i = __ffs(more) - 1;
+                more &= more - 1;
+                const int64_t ra = (int64_t)__shfl_sync(0xffffffffu, my_a, i) + W;
+                const int64_t rb = (int64_t)__shfl_sync(0xffffffffu, my_e, i);
+                double tot = 0.0, acc[8];
+#pragma unroll
+                for (int q = 0; q < 8; ++q) acc[q] = 0.0;
+                int it = 0;
+                int64_t k = ra + lane;
+                for (; k + 7 * 32 < rb; k += 8 * 32) {
+                    int d[8];
+                    V w[8];
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
+                    if (++it == kFold) {                 // blocked summation (A13)
+#pragma unroll
+                        for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
+                        it = 0;
                     }
                 }
-                mine = s[0];
+                for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ldx<HOT>(x, xh, ld_hint(col + k, pa), px);
+                double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
+                part = warp_sum(tot + part);
+                const int writer = (i / U) * W + i % U;   // lane holding row i's group sum
+                if (lane == writer) mine += part;
             }
-            // rows longer than W: the remainder is processed by the WHOLE warp, one row at a
-            // time (the paper's warp-per-row vector kernel), 8 loads per lane in
-            // flight, accumulators folded every kFold steps (A13); lane i holds row i's range
-            {
-                // lane i's row range, derived only here: contiguous batches hold row starts
-                // (the batch end in rhi), compacted ones hold [start, end) directly
-                const IT my_a = ra0;
-                const IT nx = __shfl_sync(0xffffffffu, ra0, (lane + 1) & 31);
-                const IT my_e = contiguous ? (lane + 1 < R ? nx : rhi) : rhi;
-                const int64_t my_len = (int64_t)my_e - (int64_t)my_a;
-                const bool is_long = slot_ok && my_len > W && (!CHUNKED || my_len <= long_len);
-                // remainders of at most kSubMax: all such rows of the batch at once, a subgroup
-                // of SW = 32 / next_pow2(count) lanes per row, 8 predicated loads per lane per
-                // step -- one gather round trip for the batch instead of one per row (R-MAT's
-                // many rows a little longer than W)
-                const unsigned few = __ballot_sync(0xffffffffu, is_long && my_len - W <= kSubMax);
-                unsigned more = __ballot_sync(0xffffffffu, is_long) & ~few;
-                if (few) {
-                    const int nl = __popc(few);
-                    const int lg = nl > 1 ? 32 - __clz(nl - 1) : 0;
-                    const int SW = 32 >> lg;
-                    const int sg = lane >> (5 - lg), sl = lane & (SW - 1);
-                    const int ri = sg < nl ? (int)__fns(few, 0, sg + 1) : 0;
-                    const int64_t ra = (int64_t)__shfl_sync(0xffffffffu, my_a, ri) + W;
-                    const int64_t re = (int64_t)__shfl_sync(0xffffffffu, my_e, ri);
-                    const int64_t rb = sg < nl ? re : ra;
-                    double acc[8];
-    #pragma unroll
-                    for (int q = 0; q < 8; ++q) acc[q] = 0.0;
-                    for (int64_t k = ra + sl; k < rb; k += 8 * SW) {
-                        int d[8];
-                        V w[8];
-    #pragma unroll
-                        for (int q = 0; q < 8; ++q) {
-                            const bool in = k + q * SW < rb;
-                            d[q] = in ? ld_hint(col + k + q * SW, pa) : -1;
-                            w[q] = in ? ld_hint(val + k + q * SW, pa) : (V)0;
-                        }
-    #pragma unroll
-                        for (int q = 0; q < 8; ++q) if (d[q] != -1) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
-                    }
-                    double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
-                    for (int o = SW >> 1; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
-                    const int wi = g * U + (sub < U ? sub : 0);           // this lane's row (writer lanes)
-                    const bool wmine = sub < U && ((few >> wi) & 1u);
-                    const int src = (__popc(few & ((1u << wi) - 1u)) << (5 - lg)) & 31;
-                    const double got = __shfl_sync(0xffffffffu, part, src);
-                    if (wmine) mine += got;
-                }
-                while (more) {
-                    const int i = __ffs(more) - 1;
-                    more &= more - 1;
-                    const int64_t ra = (int64_t)__shfl_sync(0xffffffffu, my_a, i) + W;
-                    const int64_t rb = (int64_t)__shfl_sync(0xffffffffu, my_e, i);
-                    double tot = 0.0, acc[8];
-    #pragma unroll
-                    for (int q = 0; q < 8; ++q) acc[q] = 0.0;
-                    int it = 0;
-                    int64_t k = ra + lane;
-                    for (; k + 7 * 32 < rb; k += 8 * 32) {
-                        int d[8];
-                        V w[8];
-    #pragma unroll
-                        for (int q = 0; q < 8; ++q) { d[q] = ld_hint(col + k + 32 * q, pa); w[q] = ld_hint(val + k + 32 * q, pa); }
-    #pragma unroll
-                        for (int q = 0; q < 8; ++q) acc[q] += (double)w[q] * (double)ldx<HOT>(x, xh, d[q], px);
-                        if (++it == kFold) {                 // blocked summation (A13)
-    #pragma unroll
-                            for (int q = 0; q < 8; ++q) { tot += acc[q]; acc[q] = 0.0; }
-                            it = 0;
-                        }
-                    }
-                    for (; k < rb; k += 32) acc[0] += (double)ld_hint(val + k, pa) * (double)ldx<HOT>(x, xh, ld_hint(col + k, pa), px);
-                    double part = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
-                    part = warp_sum(tot + part);
-                    const int writer = (i / U) * W + i % U;   // lane holding row i's group sum
-                    if (lane == writer) mine += part;
-                }
-            }
-            if (sub < U && row_ok) {
-                double o = alpha * mine;
-                if (!B0) o = fma(beta, yv, o);
-                y[my_row] = (V)o;
-            }
+        }
+        if (sub < U && row_ok) {
+            double o = alpha * mine;
+            if (!B0) o = fma(beta, yv, o);
+            y[my_row] = (V)o;
+        }
     };
     // DYN: warps take work from a global counter (zeroed before the launch), the next
     // claim requested one claim ahead -- balances skewed rows (a static grid stride left
