@@ -371,6 +371,9 @@ spmv_status convert_t(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, const s
             SPMV_LAUNCH_CHECK();
         }
         h->n_carry = ceil_div<int64_t>(nnz, kCooItems);
+        // persistent tiles for regular matrices in fp64 (no empty row, rows of at most 32;
+        // spmv_kernels.cu k_coo PERSIST)
+        h->coo_persist = sizeof(V) == 8 && fs.n_empty == 0 && fs.len_max <= 32 && n > 0;
         break;
     }
     case SPMV_ELL: {
@@ -587,6 +590,7 @@ spmv_status convert_impl(spmv_ctx *ctx, spmv_format fmt, const spmv_csr *A, cons
         }
         fs = FeatureSums{};
         fs.len_max = (unsigned long long)f->nnz_max;
+        fs.n_empty = (unsigned long long)f->n_empty_rows;
         fs.hyb_coo_ceil = (unsigned long long)f->hyb_coo_nnz;
         cusp = f->hyb_width_cusp;
     } else {

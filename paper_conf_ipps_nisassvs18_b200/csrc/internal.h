@@ -81,6 +81,7 @@ struct spmv_handle {
     int64_t sigma = 0, n_tiles = 0, map_len = 0;
     int64_t csr5_tail_row = 0;     // first row starting in the CSR5 tail (host copy of row_lo[n_tiles])
     int64_t merge_T = 0, merge_tiles = 0, merge_lean = 0;   // merge_lean: class-1 tiles (A28)
+    bool coo_persist = false;                // COO: persistent tile loop (regular matrix, fp64)
     int64_t vec_w = 0;
     int64_t csr_chunk = 0, csr_chunks = 0;   // CSR long-row split (A25): chunk length, chunk count
     // per-run scratch: carries (row, value) of CTAs/tiles for the fix-up pass
